@@ -1,0 +1,495 @@
+#!/usr/bin/env python
+"""bench.py -- params updated/sec of the AGO AdamW step on B200.
+
+One "step" = one pass of the whole hot path over the model
+states: ratel_adam_step(t), one ratel_offload_grad_chunk per block in
+decreasing block order (the order backward produces them, PAPER.md
+P:L1038-1041), ratel_sync.  Default workload at N=1: BASELINE.json
+configs[1], the 13B GPT model states of Table IV resident in
+HBM.  With N>1 (torchrun) the same 13B states are range-sharded over the
+ranks (strong scaling) with the per-block bf16 all-gather over NCCL.
+
+Printed: ONE JSON line on rank 0.
+  value      params/s over the timed region (device clock, max over ranks)
+  e2e        same metric through the C ABI with HOST buffers: states in
+             pinned host memory streamed by the library's tile ring, grads
+             H2D from pinned host and P16 D2H, all inside the timed region
+  roofline   the update kernel K1: 28 algorithmic B/param / its event-timed
+             launch durations vs MEASURED_PEAKS.json hbm_gbs
+  cpu_baseline  the CPU oracle on a bounded sample, on this host's cores
+`--impl reference` times the oracle as the reference arm.
+"""
+from __future__ import annotations
+
+import argparse
+import datetime
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+if ROOT not in sys.path:
+    sys.path.insert(0, ROOT)
+
+METRIC = "params updated/sec (Adam step) and % of HBM / host-link roofline at 1/2/4/8 B200"
+UNIT = "params/s"
+VOCAB, SEQ = 50257, 1024
+# Table IV: name -> (layers, hidden)
+SHAPES = {"c1": (1, 256), "13B": (40, 5120), "30B": (48, 7168), "70B": (80, 8192), "175B": (96, 12288)}
+HP = dict(lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, weight_decay=1e-2)   # torch defaults (R14)
+BYTES_PER_PARAM = 28                        # g 2 + theta/m/v 12 read; theta/m/v 12 + p 2 write
+
+
+def block_params(h: int) -> int:
+    return 12 * h * h + 13 * h
+
+
+def embed_params(h: int) -> int:
+    return VOCAB * h + SEQ * h + 2 * h
+
+
+def model_blocks(shape: str, with_embedding: bool = True):
+    L, h = SHAPES[shape]
+    sizes = [block_params(h)] * L
+    if with_embedding and shape != "c1":
+        sizes.append(embed_params(h))      # handed off last (R10)
+    return sizes
+
+
+# --------------------------------------------------------------- helpers
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def ncu_traffic_per_param():
+    """dram bytes per param of K1 from the committed ncu summary, if any."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "k1_ncu_summary.json")) as f:
+            return float(json.load(f)["dram_bytes_per_param"])
+    except Exception:
+        return None
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+
+    def __init__(self, gpu_id: str):
+        self.samples = []
+        self.window = None
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                       "-i", gpu_id, "-lms", "100"], stdout=subprocess.PIPE,
+                                      stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.p = None
+
+    def _read(self):
+        for line in self.p.stdout:
+            self.samples.append((time.time(), [x.strip() for x in line.split(",")]))
+
+    def mark(self, t0, t1):
+        self.window = (t0, t1)
+
+    def stop(self):
+        if self.p is None:
+            return None
+        time.sleep(0.25)
+        self.p.terminate()
+        try:
+            self.p.wait(timeout=5)
+        except Exception:
+            self.p.kill()
+        t0, t1 = self.window or (0, 1e30)
+        rows = [r for (t, r) in self.samples if t0 - 0.05 <= t <= t1 + 0.15 and len(r) >= 7]
+        if not rows:
+            rows = [r for (_, r) in self.samples if len(r) >= 7][-3:]
+        if not rows:
+            return None
+        sm = sorted(float(r[0]) for r in rows if r[0].replace(".", "").isdigit())
+        reasons = sorted({self.NAMES[i] for r in rows for i in range(4) if r[3 + i].lower() == "active"})
+        return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": float(rows[0][1]),
+                "reasons": reasons, "samples": len(rows)}
+
+
+def gpu_uuid(torch, dev):
+    try:
+        return "GPU-" + str(torch.cuda.get_device_properties(dev).uuid)
+    except Exception:
+        return str(dev)
+
+
+# ------------------------------------------------------ reference arm (oracle)
+def oracle_sample_rate(n: int, steps: int, threads: int, min_seconds: float = 0.0):
+    """Time the CPU oracle's update over an n-element sample of block 0 of the
+    workload (inputs generated outside the timed region)."""
+    import numpy as np
+    import oracle
+    import synth
+    r = oracle.Range.fresh(synth.theta0(n, block=0))
+    r.theta_bar = r.m_bar = None
+    grads = [synth.grad16(n, step=t, block=0) for t in range(1, 3)]
+    oracle.adam_range(r, grads[0], oracle.hparams(step=1), threads=threads)  # warm / first-touch
+    done, t0, t = 0, time.perf_counter(), 2
+    while done < steps or (time.perf_counter() - t0) < min_seconds:
+        oracle.adam_range(r, grads[t % 2], oracle.hparams(step=t), threads=threads)
+        done += 1
+        t += 1
+    dt = time.perf_counter() - t0
+    return n * done / dt, done, dt
+
+
+def host_threads():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    n = args.oracle_sample
+    threads = host_threads()
+    steps = args.steps
+    # warmup steps: untimed oracle passes
+    oracle_sample_rate(n, max(1, args.warmup), threads)
+    v, done, dt = oracle_sample_rate(n, steps, threads)
+    cfg = workload_config(args, world)
+    sample = (f"{n:,} params of block 0 of the {cfg['workload']} (one 13B-block slice), "
+              f"{done} steps, {threads} threads")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+        "steps": done, "warmup": args.warmup, "ms_per_step": 1e3 * dt / done * (cfg["params"] / n),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic", "config": cfg,
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+# --------------------------------------------------------------- workload
+def workload_config(args, world):
+    shape = args.shape
+    sizes = model_blocks(shape)
+    if args.blocks:
+        sizes = sizes[:args.blocks]
+    P = sum(sizes)
+    resid = "pinned-host" if args.residency == "host" else "device"
+    name = {"13B": "13B", "30B": "30B", "70B": "70B (Table IV shape, 64.9B)", "175B": "175B",
+            "c1": "C1 tiny block"}[shape]
+    return {"workload": f"{name} GPT model states ({len(sizes)} blocks), {resid}-resident, AdamW, "
+                        f"per-block AGO hand-off" + (", clip" if args.clip > 0 else ""),
+            "params": P, "blocks": len(sizes), "block_params": sizes[0], "residency": resid,
+            "parallelism": f"range-sharded x{world}" if world > 1 else "single GPU",
+            "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
+            "max_grad_norm": args.clip}
+
+
+class Model:
+    """Synthetic model states of one rank: per block one flat range."""
+
+    def __init__(self, R, torch, dev, sizes, world, rank, residency, grad_ring=2, pin_grads=False):
+        self.sizes = sizes
+        self.ranges = []
+        self.keep = []
+        self.slices = []
+        cap_max = max(R.ratel_padded_numel(n, world) for n in sizes)
+        self.grad_ring = [torch.empty(cap_max, dtype=torch.bfloat16, device=dev) for _ in range(grad_ring)]
+        for i, g in enumerate(self.grad_ring):
+            key = R.ratel_gen_stream_key(0x5EED5EED, 2, 1, i)
+            R.ratel_gen_grad16(g.data_ptr(), cap_max, 0, key)
+        self.p16 = []
+        for b, n in enumerate(sizes):
+            cap = R.ratel_padded_numel(n, world)
+            beg, end = R.ratel_rank_slice(n, world, rank)
+            s = max(end - beg, 8)
+            p = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+            if residency == "device":
+                th = torch.empty(s, dtype=torch.float32, device=dev)
+                m = torch.zeros(s, dtype=torch.float32, device=dev)
+                v = torch.zeros(s, dtype=torch.float32, device=dev)
+                R.ratel_gen_theta0(th.data_ptr(), end - beg, beg, R.ratel_gen_stream_key(0x5EED5EED, 1, 0, b))
+            else:
+                tmp = torch.empty(s, dtype=torch.float32, device=dev)
+                R.ratel_gen_theta0(tmp.data_ptr(), end - beg, beg, R.ratel_gen_stream_key(0x5EED5EED, 1, 0, b))
+                th = torch.empty(s, dtype=torch.float32, pin_memory=True)
+                th.copy_(tmp)
+                del tmp
+                m = torch.zeros(s, dtype=torch.float32, pin_memory=True)
+                v = torch.zeros(s, dtype=torch.float32, pin_memory=True)
+            g = self.grad_ring[b % grad_ring]
+            self.ranges.append(R.make_range(p, g, th, m, v, n))
+            self.keep.append((p, th, m, v))
+            self.p16.append(p)
+            self.slices.append((beg, end))
+        torch.cuda.synchronize()
+
+
+def init_lib(R, torch, dev_index, rank, world, cfg):
+    uid = None
+    if world > 1:
+        import torch.distributed as dist
+        buf = torch.zeros(128, dtype=torch.uint8, device=f"cuda:{dev_index}")
+        if rank == 0:
+            buf.copy_(torch.frombuffer(bytearray(R.ratel_get_nccl_unique_id()), dtype=torch.uint8))
+        dist.broadcast(buf, 0)
+        uid = bytes(buf.cpu().numpy().tobytes())
+    R.ratel_init(dev_index, rank, world, uid, cfg)
+
+
+def step_once(R, t, order, stream):
+    R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
+    for b in order:
+        R.ratel_offload_grad_chunk(b, stream)
+    R.ratel_sync(stream)
+
+
+def timed_steps(R, torch, order, stream, t0, K, pre_step=None, post_step=None):
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ev0.record(stream)
+    for k in range(K):
+        if pre_step:
+            pre_step(k)
+        step_once(R, t0 + k, order, stream)
+        if post_step:
+            post_step(k)
+    ev1.record(stream)
+    ev1.synchronize()
+    return ev0.elapsed_time(ev1)
+
+
+def max_over_ranks(torch, x, world, dev):
+    if world == 1:
+        return x
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def barrier(torch, world):
+    torch.cuda.synchronize()
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.synchronize()
+
+
+# ------------------------------------------------------------------- e2e
+def run_e2e(args, R, torch, dev, dev_index, rank, world):
+    """Pinned-host residency through the C ABI: theta/m/v stream H2D/D2H via
+    the library's tile ring; grads H2D from pinned host before each block's
+    hand-off; P16 D2H after the sync -- all inside the timed region."""
+    L, h = SHAPES[args.shape]
+    n_blk = args.e2e_blocks
+    sizes = [block_params(h)] * n_blk
+    cfg = R.ratel_default_config()
+    cfg.timing = 0
+    init_lib(R, torch, dev_index, rank, world, cfg)
+    try:
+        model = Model(R, torch, dev, sizes, world, rank, "host", grad_ring=1)
+        # host-side grads (one pinned buffer, re-sent for every block) and P16 out
+        cap = model.grad_ring[0].numel()
+        g_host = torch.empty(cap, dtype=torch.bfloat16, pin_memory=True)
+        g_host.copy_(model.grad_ring[0])
+        g_dev = [torch.empty(cap, dtype=torch.bfloat16, device=dev) for _ in range(n_blk)]
+        for b in range(n_blk):
+            model.ranges[b].grad_bf16 = g_dev[b].data_ptr()
+        model.grad_ring = None
+        p_host = [torch.empty(R.ratel_padded_numel(n, world), dtype=torch.bfloat16, pin_memory=True)
+                  for n in sizes]
+        for b in range(n_blk):
+            R.ratel_register_block(b, [model.ranges[b]], R.RATEL_PINNED_HOST)
+        s = torch.cuda.Stream(device=dev)
+        order = list(reversed(range(n_blk)))
+
+        def one_safe(t):
+            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
+            with torch.cuda.stream(s):
+                for b in order:
+                    g_dev[b].copy_(g_host, non_blocking=True)          # G16 host -> device
+                    R.ratel_offload_grad_chunk(b, s)
+            R.ratel_sync(s)
+            with torch.cuda.stream(s):
+                for b in range(n_blk):
+                    p_host[b].copy_(model.p16[b], non_blocking=True)  # P16 device -> host
+        t = 1
+        for _ in range(max(1, min(args.warmup, 2))):
+            one_safe(t)
+            t += 1
+        barrier(torch, world)
+        ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ev0.record(s)
+        K = args.e2e_steps
+        for _ in range(K):
+            one_safe(t)
+            t += 1
+        ev1.record(s)
+        ev1.synchronize()
+        ms = max_over_ranks(torch, ev0.elapsed_time(ev1), world, dev)
+        barrier(torch, world)
+        P = sum(sizes)
+        own = sum(e - b for (b, e) in model.slices)
+        h2d = (12 * own + 2 * own) * world            # states in + grads in (all ranks)
+        d2h = (12 * own) * world + 2 * sum(R.ratel_padded_numel(n, world) for n in sizes) * world
+        val = P * K / (ms / 1e3)
+        res = {"value": val, "unit": UNIT, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
+               "ms_per_step": ms / K, "steps": K, "params": P, "blocks": n_blk,
+               "host_link_gbs": (h2d + d2h) / world / (ms / K / 1e3) / 1e9,
+               "path": "pinned-host states (tile ring depth %d, %d-elem tiles)" % (cfg.pipeline_depth,
+                                                                                   cfg.tile_elems)}
+        del model
+        return res
+    finally:
+        R.ratel_finalize()
+
+
+# ------------------------------------------------------------------- main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ratel", choices=["ratel", "reference"])
+    ap.add_argument("--shape", default="13B", choices=list(SHAPES))
+    ap.add_argument("--blocks", type=int, default=0, help="use only the first N blocks")
+    ap.add_argument("--residency", default="device", choices=["device", "host"])
+    ap.add_argument("--clip", type=float, default=0.0)
+    ap.add_argument("--max-ctas", type=int, default=0)
+    ap.add_argument("--e2e-blocks", type=int, default=4)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--oracle-sample", type=int, default=1 << 25)
+    args = ap.parse_args()
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.steps < 1 or args.warmup < 0:
+        raise SystemExit("need --steps >= 1")
+
+    if args.impl == "reference":
+        if world > 1:
+            import torch.distributed as dist
+            dist.init_process_group("gloo")
+        run_reference(args, rank, world)
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+        return
+
+    import torch
+    import paper_conf_icde_liaosyxcyww25_b200 as R
+    torch.cuda.set_device(local)
+    dev = torch.device(f"cuda:{local}")
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+
+    cfgd = workload_config(args, world)
+    sizes = model_blocks(args.shape)
+    if args.blocks:
+        sizes = sizes[:args.blocks]
+    cfg = R.ratel_default_config()
+    cfg.timing = 1
+    cfg.max_ctas = args.max_ctas
+    cfg.max_grad_norm = args.clip
+    init_lib(R, torch, local, rank, world, cfg)
+    sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
+    try:
+        model = Model(R, torch, dev, sizes, world, rank, args.residency)
+        res = R.RATEL_PINNED_HOST if args.residency == "host" else R.RATEL_DEVICE
+        for b in range(len(sizes)):
+            R.ratel_register_block(b, [model.ranges[b]], res)
+        s = torch.cuda.Stream(device=dev)
+        order = list(reversed(range(len(sizes))))          # decreasing index
+        t = 1
+        for _ in range(args.warmup):
+            step_once(R, t, order, s)
+            t += 1
+        barrier(torch, world)
+        R.ratel_kernel_timing(reset=True)
+        l0 = R.ratel_launch_count()
+        w0 = time.time()
+        ms = timed_steps(R, torch, order, s, t, args.steps)
+        w1 = time.time()
+        launches = R.ratel_launch_count() - l0
+        k1_ms, k1_n = R.ratel_kernel_timing(reset=True)
+        if sampler:
+            sampler.mark(w0, w1)
+        ms = max_over_ranks(torch, ms, world, dev)
+        barrier(torch, world)
+        own = sum(e - b for (b, e) in model.slices)
+        P = sum(sizes)
+        value = P * args.steps / (ms / 1e3)
+        peak, peak_kind = peaks()
+        k1_bytes = BYTES_PER_PARAM * own * args.steps
+        achieved = k1_bytes / (k1_ms / 1e3) / 1e9 if k1_ms > 0 else None
+        tpp = ncu_traffic_per_param()
+        per_launch = own * args.steps / max(k1_n, 1)
+        roof = {"bound": "hbm", "kernel": "adam_update_kernel (K1)", "achieved": achieved, "peak": peak,
+                "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
+                "traffic": (tpp * per_launch) if tpp else None,
+                "algorithmic_bytes_per_launch": BYTES_PER_PARAM * per_launch,
+                "launches": k1_n, "avg_launch_ms": k1_ms / max(k1_n, 1),
+                "k1_share_of_step": (k1_ms / args.steps) / (ms / args.steps),
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
+        del model
+        R.ratel_finalize()
+        torch.cuda.empty_cache()
+        clocks = sampler.stop() if sampler else None
+
+        e2e = None
+        if not args.no_e2e:
+            try:
+                e2e = run_e2e(args, R, torch, dev, local, rank, world)
+            except Exception as ex:  # report, do not hide
+                e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:300],
+                       "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
+            torch.cuda.empty_cache()
+
+        cpu = None
+        if rank == 0 and world == 1 and not args.no_cpu_baseline:
+            n = args.oracle_sample
+            threads = host_threads()
+            v, done, dt = oracle_sample_rate(n, 2, threads, min_seconds=8.0)
+            cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
+                   "sample": f"{n:,} params (slice of block 0), {done} steps in {dt:.1f} s, "
+                             f"OpenMP {threads} threads"}
+
+        if rank == 0:
+            line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+                    "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
+                    "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                    "config": cfgd, "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                    "clocks": clocks, "gpu_launches": launches,
+                    "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
+            print(json.dumps(line), flush=True)
+    finally:
+        try:
+            R.ratel_finalize()
+        except Exception:
+            pass
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

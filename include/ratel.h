@@ -1,0 +1,202 @@
+/*
+ * ratel.h -- C ABI of the B200-native active-gradient-offloading optimizer step.
+ *
+ * What the library does (PAPER.md = /root/reference/PAPER.md, "P:Lnnn"):
+ *   Ratel's "active gradient offloading" (AGO, §IV-C) runs the
+ *   optimizer handler for a transformer block as soon as that block's 16-bit
+ *   gradient G16 arrives, "with a decreasing index during the backward stage"
+ *   (P:L1038-1041), instead of as a separate stage after backward (the
+ *   ZeRO-Infinity schedule).  The handler updates the
+ *   fp32 master weights P32 and the Adam states OS32 (m, v) and "produces a
+ *   16-bit parameter copy" P16 (sizes Table II);
+ *   the paper runs it as a CPU Adam.  Here the
+ *   handler is a fused sm_100a AdamW kernel launched on a dedicated optimizer
+ *   stream ordered after the backward stream by a CUDA event, with the states
+ *   either resident in HBM or held in pinned host memory and streamed through
+ *   a ring of device tiles (the paper's Fig. 3b pipeline, with
+ *   the host link in place of the SSD link).  AGO "keeps synchronous model
+ *   updating" (footnote 4 P:L1147-1152): the result is
+ *   identical to one synchronous Adam(W) step applied after backward.
+ *
+ * Update rule (the paper never writes it; it cites Adam [44], and
+ * shows torch.optim.Adam(), Fig. 4).  DESIGN.md readings:
+ *   g = fp32(G16) [* clip coef]
+ *   RATEL_ADAMW  : theta *= (1 - lr*wd)          (decoupled decay, default)
+ *   RATEL_ADAM_L2: g += wd*theta                 (torch.optim.Adam's decay)
+ *   m = b1*m + (1-b1)*g ; v = b2*v + (1-b2)*g^2
+ *   theta -= lr/(1-b1^t) * m / (sqrt(v)/sqrt(1-b2^t) + eps)
+ *   P16 = bf16_rne(theta)  (from the stored fp32 master)
+ * fp32 math (explicit FMA placement, IEEE sqrt/div, no fast-math).
+ *
+ * Call protocol (one host thread per process, one process per GPU; not
+ * re-entrant):
+ *   ratel_init -> ratel_register_block* ->
+ *     { ratel_adam_step(t) and ratel_offload_grad_chunk(b) for EVERY
+ *       registered b, in any interleaving -> ratel_sync }* -> ratel_finalize
+ *   A block's update is enqueued by whichever of ratel_adam_step(t) and its
+ *   ratel_offload_grad_chunk() arrives second: arming before backward gives
+ *   the paper's overlapped AGO, arming after all hand-offs gives the
+ *   "Ratel+ZeRO" deferred baseline.  With max_grad_norm > 0
+ *   every update waits for the last hand-off of the step (global norm).
+ *
+ * Ownership: every pointer registered is BORROWED (allocated by the caller,
+ * e.g. torch) and must stay valid and unmoved until ratel_finalize.  Between
+ * a block's hand-off and ratel_sync the caller must not touch that block's
+ * master/exp_avg/exp_avg_sq/param nor overwrite its grad (in torch:
+ * grad.record_stream(ratel_optimizer_stream())).  The library owns only what
+ * it creates: streams, events, device tiles, reduction buffers, NCCL comm.
+ *
+ * Errors: every int-returning call returns RATEL_OK (0) or a negative code.
+ * RATEL_EINVAL / RATEL_ESTATE have no side effects.  A CUDA or NCCL failure
+ * (including an asynchronous one detected later) is STICKY: every later call
+ * returns it until ratel_finalize.  ratel_last_error() gives a thread-local
+ * message for the last failure.
+ */
+#ifndef RATEL_H
+#define RATEL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RATEL_ABI_VERSION 1
+#define RATEL_MAX_BLOCKS 4096          /* block ids are 0 .. RATEL_MAX_BLOCKS-1 */
+#define RATEL_MAX_RANGES_PER_BLOCK 32
+
+enum {
+  RATEL_OK = 0,
+  RATEL_EINVAL = -1,     /* bad argument (pointer kind, alignment, size, value) */
+  RATEL_ESTATE = -2,     /* call out of protocol order */
+  RATEL_ECUDA = -3,      /* CUDA runtime failure (sticky) */
+  RATEL_ENCCL = -4,      /* NCCL failure (sticky) */
+  RATEL_ENOMEM = -5,     /* device/host allocation failed (sticky) */
+  RATEL_ENONFINITE = -6  /* clip mode: global grad norm was NaN/Inf (update still applied, like torch) */
+};
+
+typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1 } ratel_residency;
+typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
+/* Pinned-host staging schedule: PIPELINED = Fig. 3b (stage-in of tile k+1,
+ * update of tile k and write-back of tile k-1 overlap on three streams);
+ * SERIALIZED = Fig. 3a (naive AGO: stage-in, update, write-back in series). */
+typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1 } ratel_staging;
+
+typedef struct {
+  int mode;               /* ratel_mode; default RATEL_ADAMW */
+  double max_grad_norm;   /* > 0 enables the global L2-norm clip (torch clip_grad_norm_); default 0 */
+  int pipeline_depth;     /* pinned-host tile ring depth, 2 or 3; default 3 */
+  int staging;            /* ratel_staging; default PIPELINED */
+  uint64_t tile_elems;    /* pinned-host tile length in elements, multiple of 8; default 1<<24 */
+  int max_ctas;           /* cap on the update kernel's grid (0 = SMs x resident CTAs) */
+  int timing;             /* 1: bracket every update-kernel launch with CUDA events (ratel_kernel_timing) */
+} ratel_config;
+
+/* One contiguous parameter range of a block (a flat tensor, or a block's
+ * whole flat parameter buffer).  Element i of the range is (param[i],
+ * grad[i], master/exp_avg/exp_avg_sq[i - slice_begin]).
+ *   param_bf16   device; the FULL range, capacity ratel_padded_numel(numel, N)
+ *                elements (pads zero); this rank writes its slice and, when
+ *                N > 1, the bf16 all-gather fills the rest in place.
+ *   grad_bf16    device; the full range, or only this rank's slice when
+ *                grad_is_rank_slice = 1 (e.g. a reduce-scatter output).
+ *   master, exp_avg, exp_avg_sq
+ *                fp32, THIS RANK'S SLICE ONLY (ratel_rank_slice), on the
+ *                device (RATEL_DEVICE) or in page-locked host memory
+ *                (RATEL_PINNED_HOST; cudaHostAlloc'd or cudaHostRegister'ed).
+ *   numel        true length of the range (> 0).
+ *   apply_weight_decay  0 exempts the range from weight decay (biases, LN).
+ * All five pointers must be 16-byte aligned. */
+typedef struct {
+  void* param_bf16;
+  const void* grad_bf16;
+  int grad_is_rank_slice;
+  float* master;
+  float* exp_avg;
+  float* exp_avg_sq;
+  uint64_t numel;
+  int apply_weight_decay;
+} ratel_range;
+
+/* Fills *cfg with the defaults listed above. */
+void ratel_default_config(ratel_config* cfg);
+
+/* Writes a 128-byte NCCL unique id (rank 0 calls it and broadcasts the bytes
+ * through the caller's process group).  RATEL_ENCCL if NCCL cannot be loaded. */
+int ratel_get_nccl_unique_id(void* out128);
+
+/* Creates the optimizer/copy/comm streams (the optimizer stream at the
+ * lowest priority), events and, for world_size > 1, the NCCL communicator.
+ * device: CUDA ordinal this process drives.  nccl_unique_id: 128 bytes, NULL
+ * when world_size == 1.  cfg: NULL = defaults.  RATEL_ESTATE if already
+ * initialised; RATEL_ECUDA if no usable device. */
+int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id,
+               const ratel_config* cfg);
+
+/* Registers block `block_id` (0 <= id < RATEL_MAX_BLOCKS, each id once) made
+ * of n_ranges (1..RATEL_MAX_RANGES_PER_BLOCK) ranges, all with the given
+ * residency (ratel_residency).  Validates pointer kinds (device pointers on
+ * this device; pinned host for RATEL_PINNED_HOST -- pageable memory is
+ * RATEL_EINVAL), alignment and sizes.  The ranges array is copied.  Not
+ * allowed while a step is in flight (RATEL_ESTATE). */
+int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, int residency);
+
+/* Arms optimizer step `step` (1-based t, strictly increasing across steps)
+ * with the given hyperparameters (0 <= beta < 1, lr, eps, wd >= 0, finite).
+ * Blocks already handed off in this step are enqueued now (deferred mode);
+ * blocks handed off later are enqueued at their hand-off (AGO). */
+int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay,
+                    int64_t step);
+
+/* "Active message" for block `block_id`: its gradient is complete on
+ * `stream` (a cudaStream_t, NULL = legacy default stream).  Records an event
+ * on `stream`; the optimizer stream waits on it -- no host blocking, no data
+ * movement.  RATEL_ESTATE if the block was already handed off this step or
+ * is not registered. */
+int ratel_offload_grad_chunk(int block_id, void* stream);
+
+/* Ends the step: `stream` (cudaStream_t) is ordered after every update,
+ * write-back and all-gather of the step, so the next forward on it reads the
+ * updated P16 (no staleness, footnote 4 P:L1147-1152).  stream == NULL
+ * blocks the host instead.  RATEL_ESTATE if the step is armed but some
+ * registered block was not handed off (or vice versa).  In clip mode a
+ * blocking sync returns RATEL_ENONFINITE if the global norm was not finite. */
+int ratel_sync(void* stream);
+
+/* Waits for outstanding work, destroys everything the library created and
+ * clears all registrations and the sticky error. */
+int ratel_finalize(void);
+
+/* Message describing the last error on this thread ("" if none). */
+const char* ratel_last_error(void);
+
+/* Capacity of a range's param buffer for world_size ranks: numel rounded up
+ * to a multiple of 8*world_size (each rank's slice is a multiple of 8
+ * elements, keeping 16-byte alignment).  Pure host function. */
+uint64_t ratel_padded_numel(uint64_t numel, int world_size);
+
+/* This rank's slice [*begin, *end) of a range of numel elements:
+ * s = ratel_padded_numel(numel, N)/N, begin = min(numel, rank*s),
+ * end = min(numel, begin + s).  Pure host function. */
+int ratel_rank_slice(uint64_t numel, int world_size, int rank, uint64_t* begin, uint64_t* end);
+
+/* The optimizer stream (cudaStream_t) -- for torch's record_stream. NULL before init. */
+void* ratel_optimizer_stream(void);
+
+/* Blocking: the global sum of squared gradients of the last clip-mode step
+ * (after the allreduce).  RATEL_ESTATE if clipping is off. */
+int ratel_get_grad_sumsq(double* out);
+
+/* Sum of the update kernel's event-timed durations (ms) and number of timed
+ * launches since the last reset (requires cfg.timing = 1; blocking). */
+int ratel_kernel_timing(double* total_ms, int64_t* launches, int reset);
+
+/* Number of kernels this library launched since init (update, grad-norm
+ * partial and finalize kernels). */
+int64_t ratel_launch_count(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RATEL_H */

@@ -1,0 +1,703 @@
+// ratel_runtime.cu -- the C ABI (include/ratel.h): registration, the per-step
+// state machine of active gradient offloading, the pinned-host tile ring, the
+// optional global-norm clip and the multi-GPU range partition.
+//
+// PAPER.md anchors: AGO's "active message" -- the optimizer handler for a
+// tensor runs "upon main memory receiving the offloaded gradients"
+// (P:L1017-1031); gradients arrive "sequentially with a decreasing index"
+// (P:L1038-1041); naive AGO serialises state-in, compute, state-out
+// (Fig. 3a) while optimized AGO overlaps the write-back of
+// tensor i with the compute of tensor i-1 (Fig. 3b).  Here the
+// "message" is a CUDA event recorded on the caller's backward stream, the
+// handler is the K1 kernel on a low-priority optimizer stream, and for
+// pinned-host states the state-in / write-back run on two copy streams (the
+// host link is duplex, unlike the paper's SSD link).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <new>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <vector>
+
+#include "nccl_dl.h"
+#include "ratel.h"
+#include "ratel_kernels.cuh"
+
+namespace {
+
+using namespace ratel;
+
+thread_local char t_err[1024] = "";
+
+int set_error(int code, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(t_err, sizeof t_err, fmt, ap);
+  va_end(ap);
+  return code;
+}
+
+struct Slice {
+  uint64_t begin = 0, end = 0;
+};
+
+struct Block {
+  bool registered = false;
+  int residency = RATEL_DEVICE;
+  int order = -1;  // registration index (fixes the clip reduction order)
+  std::vector<ratel_range> ranges;
+  std::vector<Slice> slices;
+  cudaEvent_t ev_grad = nullptr;  // "gradient arrived" -- recorded on the caller's stream
+  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt
+  bool handed_off = false, enqueued = false;
+};
+
+struct TimingPair {
+  cudaEvent_t a = nullptr, b = nullptr;
+};
+
+struct Ctx {
+  bool inited = false;
+  int sticky = 0;
+  char sticky_msg[1024] = "";
+  int device = 0, rank = 0, world = 1;
+  ratel_config cfg{};
+  int sms = 0, k1_grid = 0, k2_grid = 0;
+  cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr;
+  cudaEvent_t ev_end[4] = {nullptr, nullptr, nullptr, nullptr};
+  std::vector<Block> blocks;
+  std::vector<int> reg;      // registered ids, registration order
+  std::vector<int> pending;  // handed off before arming (deferred), hand-off order
+  int n_handed = 0;
+  bool armed = false;
+  int64_t last_step = 0;
+  AdamScalars scal{};
+  // clip
+  double* d_partials = nullptr;
+  size_t partial_cap = 0;  // slots
+  double* d_sumsq = nullptr;  // [0] this rank, [1] all ranks
+  int* h_flag = nullptr;      // mapped pinned: non-finite norm seen
+  int* d_flag = nullptr;
+  // pinned-host tile ring
+  float* d_tiles = nullptr;  // depth x {theta, m, v} x tile
+  cudaEvent_t ev_h2d[3] = {}, ev_k1[3] = {}, ev_d2h[3] = {};
+  uint64_t ring_k = 0;
+  // NCCL
+  ncclComm_t comm = nullptr;
+  // stats
+  int64_t launches = 0;
+  std::vector<TimingPair> tpool;
+  size_t tused = 0;
+};
+
+Ctx G;
+NcclApi g_nccl;
+
+int sticky_fail(int code, const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(G.sticky_msg, sizeof G.sticky_msg, fmt, ap);
+  va_end(ap);
+  G.sticky = code;
+  snprintf(t_err, sizeof t_err, "%s", G.sticky_msg);
+  return code;
+}
+
+#define CK(call)                                                                                 \
+  do {                                                                                           \
+    cudaError_t e_ = (call);                                                                     \
+    if (e_ != cudaSuccess)                                                                       \
+      return sticky_fail(e_ == cudaErrorMemoryAllocation ? RATEL_ENOMEM : RATEL_ECUDA,           \
+                         "%s failed: %s (%s:%d)", #call, cudaGetErrorString(e_), __FILE__, __LINE__); \
+  } while (0)
+
+#define NK(call)                                                                                  \
+  do {                                                                                            \
+    ncclResult_t r_ = (call);                                                                     \
+    if (r_ != ncclSuccess)                                                                        \
+      return sticky_fail(RATEL_ENCCL, "%s failed: %s (%s:%d)", #call, g_nccl.GetErrorString(r_), \
+                         __FILE__, __LINE__);                                                     \
+  } while (0)
+
+#define RK(call)              \
+  do {                        \
+    int rc_ = (call);         \
+    if (rc_ != RATEL_OK) return rc_; \
+  } while (0)
+
+int entry() {
+  if (!G.inited) return set_error(RATEL_ESTATE, "ratel: not initialised (call ratel_init first)");
+  if (G.sticky) return set_error(G.sticky, "ratel: sticky error: %s", G.sticky_msg);
+  CK(cudaSetDevice(G.device));
+  return RATEL_OK;
+}
+
+uint64_t padded(uint64_t n, int world) {
+  const uint64_t q = 8ull * static_cast<uint64_t>(world);
+  return (n + q - 1) / q * q;
+}
+
+Slice slice_of(uint64_t n, int world, int rank) {
+  const uint64_t s = padded(n, world) / world;
+  Slice r;
+  r.begin = std::min<uint64_t>(n, s * rank);
+  r.end = std::min<uint64_t>(n, r.begin + s);
+  return r;
+}
+
+const uint16_t* grad_ptr(const ratel_range& r, const Slice& s) {
+  return static_cast<const uint16_t*>(r.grad_bf16) + (r.grad_is_rank_slice ? 0 : s.begin);
+}
+
+// ------------------------------------------------------------------ launches
+template <int MODE, bool CLIP>
+void launch_k1(const UpdateParams& P, unsigned grid) {
+  adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, G.s_opt>>>(P);
+}
+
+int launch_update(const RangeDesc* rd, int nr) {
+  if (nr == 0) return RATEL_OK;
+  UpdateParams P{};
+  uint64_t max8 = 0;
+  for (int i = 0; i < nr; ++i) {
+    P.r[i] = rd[i];
+    max8 = std::max<uint64_t>(max8, (rd[i].n + 7) / 8);
+  }
+  P.nr = nr;
+  P.s = G.scal;
+  const bool clip = G.cfg.max_grad_norm > 0.0;
+  P.sumsq = G.world > 1 ? G.d_sumsq + 1 : G.d_sumsq;
+  P.max_norm = G.cfg.max_grad_norm;
+  P.nonfinite_flag = G.d_flag;
+  const uint64_t want = std::max<uint64_t>(1, (max8 + kThreads - 1) / kThreads);
+  const unsigned grid = static_cast<unsigned>(std::min<uint64_t>(want, static_cast<uint64_t>(G.k1_grid)));
+  TimingPair* tp = nullptr;
+  if (G.cfg.timing) {
+    if (G.tused == G.tpool.size()) {
+      TimingPair t;
+      CK(cudaEventCreate(&t.a));
+      CK(cudaEventCreate(&t.b));
+      G.tpool.push_back(t);
+    }
+    tp = &G.tpool[G.tused++];
+    CK(cudaEventRecord(tp->a, G.s_opt));
+  }
+  if (G.cfg.mode == RATEL_ADAMW)
+    clip ? launch_k1<RATEL_ADAMW, true>(P, grid) : launch_k1<RATEL_ADAMW, false>(P, grid);
+  else
+    clip ? launch_k1<RATEL_ADAM_L2, true>(P, grid) : launch_k1<RATEL_ADAM_L2, false>(P, grid);
+  CK(cudaGetLastError());
+  ++G.launches;
+  if (tp) CK(cudaEventRecord(tp->b, G.s_opt));
+  return RATEL_OK;
+}
+
+int launch_sumsq(const Block& B) {
+  SumsqParams S{};
+  int nr = 0;
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const Slice& s = B.slices[i];
+    if (s.end == s.begin) continue;
+    S.g[nr] = grad_ptr(B.ranges[i], s);
+    S.n[nr] = s.end - s.begin;
+    ++nr;
+  }
+  S.nr = nr;
+  S.partials = G.d_partials + static_cast<size_t>(B.order) * G.k2_grid;
+  grad_sumsq_kernel<<<G.k2_grid, kThreads, 0, G.s_opt>>>(S);
+  CK(cudaGetLastError());
+  ++G.launches;
+  return RATEL_OK;
+}
+
+// One staged tile of a pinned-host range: H2D(theta, m, v) -> K1 -> D2H.
+int stage_tile(const ratel_range& r, const Slice& s, uint64_t off, uint64_t len) {
+  const int k = static_cast<int>(G.ring_k % static_cast<uint64_t>(G.cfg.pipeline_depth));
+  const uint64_t T = G.cfg.tile_elems;
+  float* th = G.d_tiles + (3ull * k + 0) * T;
+  float* m = G.d_tiles + (3ull * k + 1) * T;
+  float* v = G.d_tiles + (3ull * k + 2) * T;
+  const size_t bytes = len * sizeof(float);
+  RangeDesc rd{};
+  rd.g = grad_ptr(r, s) + off;
+  rd.th = th;
+  rd.m = m;
+  rd.v = v;
+  rd.p = static_cast<uint16_t*>(r.param_bf16) + s.begin + off;
+  rd.n = len;
+  rd.wd_on = r.apply_weight_decay != 0;
+  const bool serial = G.cfg.staging == RATEL_STAGING_SERIALIZED;
+  cudaStream_t in = serial ? G.s_opt : G.s_h2d;
+  cudaStream_t out = serial ? G.s_opt : G.s_d2h;
+  if (!serial && G.ring_k >= static_cast<uint64_t>(G.cfg.pipeline_depth))
+    CK(cudaStreamWaitEvent(in, G.ev_d2h[k], 0));  // slot free: its previous write-back done
+  CK(cudaMemcpyAsync(th, r.master + off, bytes, cudaMemcpyHostToDevice, in));
+  CK(cudaMemcpyAsync(m, r.exp_avg + off, bytes, cudaMemcpyHostToDevice, in));
+  CK(cudaMemcpyAsync(v, r.exp_avg_sq + off, bytes, cudaMemcpyHostToDevice, in));
+  if (!serial) {
+    CK(cudaEventRecord(G.ev_h2d[k], in));
+    CK(cudaStreamWaitEvent(G.s_opt, G.ev_h2d[k], 0));
+  }
+  RK(launch_update(&rd, 1));
+  if (!serial) {
+    CK(cudaEventRecord(G.ev_k1[k], G.s_opt));
+    CK(cudaStreamWaitEvent(out, G.ev_k1[k], 0));
+  }
+  CK(cudaMemcpyAsync(r.master + off, th, bytes, cudaMemcpyDeviceToHost, out));
+  CK(cudaMemcpyAsync(r.exp_avg + off, m, bytes, cudaMemcpyDeviceToHost, out));
+  CK(cudaMemcpyAsync(r.exp_avg_sq + off, v, bytes, cudaMemcpyDeviceToHost, out));
+  if (!serial) CK(cudaEventRecord(G.ev_d2h[k], out));
+  ++G.ring_k;
+  return RATEL_OK;
+}
+
+int allgather_block(const Block& B) {
+  CK(cudaStreamWaitEvent(G.s_comm, B.ev_done, 0));
+  NK(g_nccl.GroupStart());
+  for (const ratel_range& r : B.ranges) {
+    const uint64_t s = padded(r.numel, G.world) / G.world;
+    uint16_t* p = static_cast<uint16_t*>(r.param_bf16);
+    NK(g_nccl.AllGather(p + s * G.rank, p, s, ncclBfloat16, G.comm, G.s_comm));
+  }
+  NK(g_nccl.GroupEnd());
+  return RATEL_OK;
+}
+
+// Enqueue the handler of block B (its s_opt wait on ev_grad was issued at
+// hand-off).  Device residency: one K1 launch over the rank's slices of all
+// ranges.  Pinned-host: the tile ring.
+int enqueue_block(Block& B) {
+  if (B.residency == RATEL_DEVICE) {
+    RangeDesc rd[kMaxRanges];
+    int nr = 0;
+    for (size_t i = 0; i < B.ranges.size(); ++i) {
+      const ratel_range& r = B.ranges[i];
+      const Slice& s = B.slices[i];
+      if (s.end == s.begin) continue;
+      RangeDesc& d = rd[nr++];
+      d.g = grad_ptr(r, s);
+      d.th = r.master;
+      d.m = r.exp_avg;
+      d.v = r.exp_avg_sq;
+      d.p = static_cast<uint16_t*>(r.param_bf16) + s.begin;
+      d.n = s.end - s.begin;
+      d.wd_on = r.apply_weight_decay != 0;
+      d.pad_ = 0;
+    }
+    RK(launch_update(rd, nr));
+  } else {
+    for (size_t i = 0; i < B.ranges.size(); ++i) {
+      const Slice& s = B.slices[i];
+      const uint64_t n = s.end - s.begin;
+      for (uint64_t off = 0; off < n; off += G.cfg.tile_elems)
+        RK(stage_tile(B.ranges[i], s, off, std::min<uint64_t>(G.cfg.tile_elems, n - off)));
+    }
+  }
+  CK(cudaEventRecord(B.ev_done, G.s_opt));
+  if (G.world > 1) RK(allgather_block(B));
+  B.enqueued = true;
+  return RATEL_OK;
+}
+
+// Clip mode: every hand-off has run K2; reduce, allreduce, then update all.
+int finalize_clip() {
+  sumsq_finalize_kernel<<<1, kThreads, 0, G.s_opt>>>(G.d_partials,
+                                                     static_cast<uint64_t>(G.reg.size()) * G.k2_grid,
+                                                     G.d_sumsq);
+  CK(cudaGetLastError());
+  ++G.launches;
+  if (G.world > 1)
+    NK(g_nccl.AllReduce(G.d_sumsq, G.d_sumsq + 1, 1, ncclFloat64, ncclSum, G.comm, G.s_opt));
+  for (int id : G.reg) RK(enqueue_block(G.blocks[id]));
+  G.pending.clear();
+  return RATEL_OK;
+}
+
+bool aligned16(const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15u) == 0; }
+
+int check_ptr(const void* p, bool want_device, const char* what, int idx) {
+  cudaPointerAttributes a{};
+  const cudaError_t e = cudaPointerGetAttributes(&a, p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_error(RATEL_EINVAL, "range %d: %s is not a CUDA-visible pointer (%s)", idx, what,
+                     cudaGetErrorString(e));
+  }
+  if (want_device) {
+    if (a.type != cudaMemoryTypeDevice || a.device != G.device)
+      return set_error(RATEL_EINVAL, "range %d: %s must be device memory on device %d", idx, what, G.device);
+  } else if (a.type != cudaMemoryTypeHost) {
+    return set_error(RATEL_EINVAL, "range %d: %s must be page-locked host memory (cudaHostAlloc/Register)",
+                     idx, what);
+  }
+  return RATEL_OK;
+}
+
+int validate_config(const ratel_config& c) {
+  if (c.mode != RATEL_ADAMW && c.mode != RATEL_ADAM_L2) return set_error(RATEL_EINVAL, "cfg.mode");
+  if (!(c.max_grad_norm >= 0.0) || !std::isfinite(c.max_grad_norm))
+    return set_error(RATEL_EINVAL, "cfg.max_grad_norm must be finite and >= 0");
+  if (c.pipeline_depth != 2 && c.pipeline_depth != 3) return set_error(RATEL_EINVAL, "cfg.pipeline_depth must be 2 or 3");
+  if (c.staging != RATEL_STAGING_PIPELINED && c.staging != RATEL_STAGING_SERIALIZED)
+    return set_error(RATEL_EINVAL, "cfg.staging");
+  if (c.tile_elems == 0 || (c.tile_elems & 7u)) return set_error(RATEL_EINVAL, "cfg.tile_elems must be a positive multiple of 8");
+  if (c.max_ctas < 0) return set_error(RATEL_EINVAL, "cfg.max_ctas must be >= 0");
+  return RATEL_OK;
+}
+
+void reset_step_state() {
+  for (int id : G.reg) {
+    G.blocks[id].handed_off = false;
+    G.blocks[id].enqueued = false;
+  }
+  G.pending.clear();
+  G.n_handed = 0;
+  G.armed = false;
+}
+
+void destroy_all() {
+  for (int id : G.reg) {
+    Block& B = G.blocks[id];
+    if (B.ev_grad) cudaEventDestroy(B.ev_grad);
+    if (B.ev_done) cudaEventDestroy(B.ev_done);
+  }
+  for (TimingPair& t : G.tpool) {
+    cudaEventDestroy(t.a);
+    cudaEventDestroy(t.b);
+  }
+  for (int k = 0; k < 3; ++k) {
+    if (G.ev_h2d[k]) cudaEventDestroy(G.ev_h2d[k]);
+    if (G.ev_k1[k]) cudaEventDestroy(G.ev_k1[k]);
+    if (G.ev_d2h[k]) cudaEventDestroy(G.ev_d2h[k]);
+  }
+  for (cudaEvent_t e : G.ev_end)
+    if (e) cudaEventDestroy(e);
+  if (G.d_tiles) cudaFree(G.d_tiles);
+  if (G.d_partials) cudaFree(G.d_partials);
+  if (G.d_sumsq) cudaFree(G.d_sumsq);
+  if (G.h_flag) cudaFreeHost(G.h_flag);
+  if (G.comm) g_nccl.CommDestroy(G.comm);
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm})
+    if (s) cudaStreamDestroy(s);
+  G.~Ctx();
+  new (&G) Ctx();
+}
+
+int init_body(int device, int rank, int world_size, const void* nccl_unique_id, const ratel_config& c) {
+  G.device = device;
+  G.rank = rank;
+  G.world = world_size;
+  G.cfg = c;
+  CK(cudaSetDevice(device));
+  cudaDeviceProp prop{};
+  CK(cudaGetDeviceProperties(&prop, device));
+  if (prop.major < 10)
+    return set_error(RATEL_ECUDA, "ratel_init: device %d is sm_%d%d; this library is built for sm_100a",
+                     device, prop.major, prop.minor);
+  G.sms = prop.multiProcessorCount;
+  int least = 0, greatest = 0;
+  CK(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_opt, cudaStreamNonBlocking, least));  // lowest priority
+  CK(cudaStreamCreateWithPriority(&G.s_h2d, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_d2h, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_comm, cudaStreamNonBlocking, greatest));
+  for (cudaEvent_t& ev : G.ev_end) CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+  for (int k = 0; k < 3; ++k) {
+    CK(cudaEventCreateWithFlags(&G.ev_h2d[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&G.ev_k1[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&G.ev_d2h[k], cudaEventDisableTiming));
+  }
+  int occ = 0;
+  if (c.mode == RATEL_ADAMW)
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, adam_update_kernel<RATEL_ADAMW, false>, kThreads, 0));
+  else
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, adam_update_kernel<RATEL_ADAM_L2, false>, kThreads, 0));
+  G.k1_grid = G.sms * std::max(occ, 1);
+  if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
+  G.k2_grid = G.sms * 2;
+  CK(cudaMalloc(&G.d_sumsq, 2 * sizeof(double)));
+  CK(cudaMemset(G.d_sumsq, 0, 2 * sizeof(double)));
+  CK(cudaHostAlloc(&G.h_flag, sizeof(int), cudaHostAllocMapped));
+  *G.h_flag = 0;
+  CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&G.d_flag), G.h_flag, 0));
+  G.blocks.assign(RATEL_MAX_BLOCKS, Block());
+  if (world_size > 1) {
+    if (const char* m = g_nccl.load()) return set_error(RATEL_ENCCL, "ratel_init: cannot load NCCL: %s", m);
+    ncclUniqueId id;
+    memcpy(&id, nccl_unique_id, sizeof id);
+    ncclComm_t comm = nullptr;
+    NK(g_nccl.CommInitRank(&comm, world_size, id, rank));
+    G.comm = comm;
+  }
+  return RATEL_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+void ratel_default_config(ratel_config* cfg) {
+  if (cfg == nullptr) return;
+  cfg->mode = RATEL_ADAMW;
+  cfg->max_grad_norm = 0.0;
+  cfg->pipeline_depth = 3;
+  cfg->staging = RATEL_STAGING_PIPELINED;
+  cfg->tile_elems = 1ull << 24;
+  cfg->max_ctas = 0;
+  cfg->timing = 0;
+}
+
+uint64_t ratel_padded_numel(uint64_t numel, int world_size) {
+  if (world_size < 1) return 0;
+  return padded(numel, world_size);
+}
+
+int ratel_rank_slice(uint64_t numel, int world_size, int rank, uint64_t* begin, uint64_t* end) {
+  if (world_size < 1 || rank < 0 || rank >= world_size || begin == nullptr || end == nullptr)
+    return set_error(RATEL_EINVAL, "ratel_rank_slice: bad arguments");
+  const Slice s = slice_of(numel, world_size, rank);
+  *begin = s.begin;
+  *end = s.end;
+  return RATEL_OK;
+}
+
+const char* ratel_last_error(void) { return t_err; }
+
+int ratel_get_nccl_unique_id(void* out128) {
+  if (out128 == nullptr) return set_error(RATEL_EINVAL, "ratel_get_nccl_unique_id: NULL");
+  if (const char* m = g_nccl.load()) return set_error(RATEL_ENCCL, "cannot load NCCL: %s", m);
+  ncclUniqueId id;
+  const ncclResult_t r = g_nccl.GetUniqueId(&id);
+  if (r != ncclSuccess) return set_error(RATEL_ENCCL, "ncclGetUniqueId: %s", g_nccl.GetErrorString(r));
+  memcpy(out128, &id, sizeof id);
+  return RATEL_OK;
+}
+
+int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id, const ratel_config* cfg) {
+  if (G.inited) return set_error(RATEL_ESTATE, "ratel_init: already initialised");
+  if (world_size < 1 || rank < 0 || rank >= world_size)
+    return set_error(RATEL_EINVAL, "ratel_init: need 0 <= rank < world_size");
+  if (world_size > 1 && nccl_unique_id == nullptr)
+    return set_error(RATEL_EINVAL, "ratel_init: world_size > 1 needs an NCCL unique id");
+  ratel_config c;
+  ratel_default_config(&c);
+  if (cfg) c = *cfg;
+  RK(validate_config(c));
+  int ndev = 0;
+  cudaError_t e = cudaGetDeviceCount(&ndev);
+  if (e != cudaSuccess || ndev == 0) {
+    cudaGetLastError();
+    return set_error(RATEL_ECUDA, "ratel_init: no CUDA device (%s)", cudaGetErrorString(e));
+  }
+  if (device < 0 || device >= ndev) return set_error(RATEL_EINVAL, "ratel_init: device %d out of range", device);
+  const int rc = init_body(device, rank, world_size, nccl_unique_id, c);
+  if (rc != RATEL_OK) {
+    char msg[1024];
+    snprintf(msg, sizeof msg, "%s", t_err);
+    destroy_all();  // also clears the sticky state: a failed init leaves nothing behind
+    cudaGetLastError();
+    return set_error(rc, "%s", msg);
+  }
+  G.inited = true;
+  t_err[0] = '\0';
+  return RATEL_OK;
+}
+
+int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, int residency) {
+  RK(entry());
+  if (G.armed || G.n_handed > 0) return set_error(RATEL_ESTATE, "ratel_register_block: a step is in flight");
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS)
+    return set_error(RATEL_EINVAL, "ratel_register_block: block id %d out of range", block_id);
+  if (G.blocks[block_id].registered)
+    return set_error(RATEL_EINVAL, "ratel_register_block: block %d already registered", block_id);
+  if (ranges == nullptr || n_ranges < 1 || n_ranges > RATEL_MAX_RANGES_PER_BLOCK)
+    return set_error(RATEL_EINVAL, "ratel_register_block: need 1..%d ranges", RATEL_MAX_RANGES_PER_BLOCK);
+  if (residency != RATEL_DEVICE && residency != RATEL_PINNED_HOST)
+    return set_error(RATEL_EINVAL, "ratel_register_block: bad residency %d", residency);
+  std::vector<Slice> slices(n_ranges);
+  for (int i = 0; i < n_ranges; ++i) {
+    const ratel_range& r = ranges[i];
+    if (r.numel == 0) return set_error(RATEL_EINVAL, "range %d: numel must be > 0", i);
+    slices[i] = slice_of(r.numel, G.world, G.rank);
+    const bool has = slices[i].end > slices[i].begin;
+    if (r.param_bf16 == nullptr || r.grad_bf16 == nullptr)
+      return set_error(RATEL_EINVAL, "range %d: param/grad pointer is NULL", i);
+    if (has && (r.master == nullptr || r.exp_avg == nullptr || r.exp_avg_sq == nullptr))
+      return set_error(RATEL_EINVAL, "range %d: state pointer is NULL", i);
+    const void* ps[5] = {r.param_bf16, r.grad_bf16, r.master, r.exp_avg, r.exp_avg_sq};
+    for (const void* p : ps)
+      if (p && !aligned16(p)) return set_error(RATEL_EINVAL, "range %d: pointers must be 16-byte aligned", i);
+    RK(check_ptr(r.param_bf16, true, "param_bf16", i));
+    RK(check_ptr(r.grad_bf16, true, "grad_bf16", i));
+    if (has) {
+      const bool dev = residency == RATEL_DEVICE;
+      RK(check_ptr(r.master, dev, "master", i));
+      RK(check_ptr(r.exp_avg, dev, "exp_avg", i));
+      RK(check_ptr(r.exp_avg_sq, dev, "exp_avg_sq", i));
+    }
+  }
+  if (residency == RATEL_PINNED_HOST && G.d_tiles == nullptr) {
+    const size_t bytes = static_cast<size_t>(G.cfg.pipeline_depth) * 3 * G.cfg.tile_elems * sizeof(float);
+    CK(cudaMalloc(&G.d_tiles, bytes));
+  }
+  if (G.cfg.max_grad_norm > 0.0) {
+    const size_t need = (G.reg.size() + 1) * static_cast<size_t>(G.k2_grid);
+    if (need > G.partial_cap) {
+      const size_t cap = std::max(need, 2 * G.partial_cap);
+      double* p = nullptr;
+      CK(cudaMalloc(&p, cap * sizeof(double)));
+      if (G.d_partials) {
+        CK(cudaMemcpy(p, G.d_partials, G.partial_cap * sizeof(double), cudaMemcpyDeviceToDevice));
+        CK(cudaFree(G.d_partials));
+      }
+      G.d_partials = p;
+      G.partial_cap = cap;
+    }
+  }
+  Block& B = G.blocks[block_id];
+  CK(cudaEventCreateWithFlags(&B.ev_grad, cudaEventDisableTiming));
+  CK(cudaEventCreateWithFlags(&B.ev_done, cudaEventDisableTiming));
+  B.ranges.assign(ranges, ranges + n_ranges);
+  B.slices = slices;
+  B.residency = residency;
+  B.order = static_cast<int>(G.reg.size());
+  B.registered = true;
+  G.reg.push_back(block_id);
+  return RATEL_OK;
+}
+
+int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay, int64_t step) {
+  RK(entry());
+  if (G.armed) return set_error(RATEL_ESTATE, "ratel_adam_step: step %lld already armed", (long long)G.last_step);
+  if (step <= G.last_step)
+    return set_error(RATEL_ESTATE, "ratel_adam_step: step %lld <= previous %lld", (long long)step,
+                     (long long)G.last_step);
+  const double vals[5] = {lr, beta1, beta2, eps, weight_decay};
+  for (double x : vals)
+    if (!std::isfinite(x) || x < 0.0) return set_error(RATEL_EINVAL, "ratel_adam_step: hyperparameters must be finite, >= 0");
+  if (beta1 >= 1.0 || beta2 >= 1.0) return set_error(RATEL_EINVAL, "ratel_adam_step: betas must be < 1");
+  const double t = static_cast<double>(step);
+  const double bc1 = 1.0 - std::pow(beta1, t);
+  const double bc2 = 1.0 - std::pow(beta2, t);
+  AdamScalars& s = G.scal;
+  s.beta1 = static_cast<float>(beta1);
+  s.one_minus_beta1 = static_cast<float>(1.0 - beta1);
+  s.beta2 = static_cast<float>(beta2);
+  s.one_minus_beta2 = static_cast<float>(1.0 - beta2);
+  s.neg_step_size = static_cast<float>(-lr / bc1);
+  s.inv_sqrt_bc2 = static_cast<float>(1.0 / std::sqrt(bc2));
+  s.eps = static_cast<float>(eps);
+  s.decay = static_cast<float>(1.0 - lr * weight_decay);
+  s.wd = static_cast<float>(weight_decay);
+  G.armed = true;
+  G.last_step = step;
+  if (G.cfg.max_grad_norm > 0.0) {
+    if (!G.reg.empty() && G.n_handed == static_cast<int>(G.reg.size())) RK(finalize_clip());
+    return RATEL_OK;
+  }
+  for (int id : G.pending) RK(enqueue_block(G.blocks[id]));  // deferred ("Ratel+ZeRO") order
+  G.pending.clear();
+  return RATEL_OK;
+}
+
+int ratel_offload_grad_chunk(int block_id, void* stream) {
+  RK(entry());
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
+    return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d is not registered", block_id);
+  Block& B = G.blocks[block_id];
+  if (B.handed_off)
+    return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d already handed off this step", block_id);
+  CK(cudaEventRecord(B.ev_grad, static_cast<cudaStream_t>(stream)));
+  CK(cudaStreamWaitEvent(G.s_opt, B.ev_grad, 0));
+  B.handed_off = true;
+  ++G.n_handed;
+  if (G.cfg.max_grad_norm > 0.0) {
+    RK(launch_sumsq(B));
+    if (G.armed && G.n_handed == static_cast<int>(G.reg.size())) RK(finalize_clip());
+    return RATEL_OK;
+  }
+  if (G.armed)
+    RK(enqueue_block(B));  // active message: handler runs now, overlapping backward
+  else
+    G.pending.push_back(block_id);
+  return RATEL_OK;
+}
+
+int ratel_sync(void* stream) {
+  RK(entry());
+  if (G.armed || G.n_handed > 0) {
+    if (!G.armed) return set_error(RATEL_ESTATE, "ratel_sync: blocks handed off but no ratel_adam_step");
+    if (G.n_handed != static_cast<int>(G.reg.size()))
+      return set_error(RATEL_ESTATE, "ratel_sync: %d of %zu blocks handed off", G.n_handed, G.reg.size());
+  }
+  cudaStream_t ss[4] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm};
+  for (int i = 0; i < 4; ++i) CK(cudaEventRecord(G.ev_end[i], ss[i]));
+  // Order the internal streams too: the next step's stage-in must not read
+  // host states still being written back, and its K1 must not overwrite a
+  // P16 slice the all-gather is still sending.
+  for (int i = 0; i < 4; ++i)
+    for (int j = 0; j < 4; ++j)
+      if (i != j) CK(cudaStreamWaitEvent(ss[i], G.ev_end[j], 0));
+  reset_step_state();
+  if (stream != nullptr) {
+    for (int i = 0; i < 4; ++i) CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), G.ev_end[i], 0));
+    CK(cudaGetLastError());
+  } else {
+    for (int i = 0; i < 4; ++i) CK(cudaEventSynchronize(G.ev_end[i]));
+  }
+  if (G.comm) {
+    ncclResult_t ar = ncclSuccess;
+    NK(g_nccl.CommGetAsyncError(G.comm, &ar));
+    if (ar != ncclSuccess && ar != ncclInProgress)
+      return sticky_fail(RATEL_ENCCL, "NCCL async error: %s", g_nccl.GetErrorString(ar));
+  }
+  if (stream == nullptr && G.cfg.max_grad_norm > 0.0 && *G.h_flag) {
+    *G.h_flag = 0;
+    return set_error(RATEL_ENONFINITE, "ratel_sync: global grad norm was not finite (update applied)");
+  }
+  return RATEL_OK;
+}
+
+int ratel_finalize(void) {
+  if (!G.inited) return set_error(RATEL_ESTATE, "ratel_finalize: not initialised");
+  cudaSetDevice(G.device);
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm})
+    if (s) cudaStreamSynchronize(s);
+  destroy_all();
+  cudaGetLastError();
+  return RATEL_OK;
+}
+
+void* ratel_optimizer_stream(void) { return G.inited ? static_cast<void*>(G.s_opt) : nullptr; }
+
+int ratel_get_grad_sumsq(double* out) {
+  RK(entry());
+  if (out == nullptr) return set_error(RATEL_EINVAL, "ratel_get_grad_sumsq: NULL");
+  if (!(G.cfg.max_grad_norm > 0.0)) return set_error(RATEL_ESTATE, "ratel_get_grad_sumsq: clipping is off");
+  CK(cudaStreamSynchronize(G.s_opt));
+  CK(cudaMemcpy(out, G.world > 1 ? G.d_sumsq + 1 : G.d_sumsq, sizeof(double), cudaMemcpyDeviceToHost));
+  return RATEL_OK;
+}
+
+int ratel_kernel_timing(double* total_ms, int64_t* launches, int reset) {
+  RK(entry());
+  if (total_ms == nullptr || launches == nullptr) return set_error(RATEL_EINVAL, "ratel_kernel_timing: NULL");
+  double tot = 0.0;
+  for (size_t i = 0; i < G.tused; ++i) {
+    CK(cudaEventSynchronize(G.tpool[i].b));
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, G.tpool[i].a, G.tpool[i].b));
+    tot += ms;
+  }
+  *total_ms = tot;
+  *launches = static_cast<int64_t>(G.tused);
+  if (reset) G.tused = 0;
+  return RATEL_OK;
+}
+
+int64_t ratel_launch_count(void) { return G.launches; }
+
+}  // extern "C"

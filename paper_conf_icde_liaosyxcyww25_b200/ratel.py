@@ -1,0 +1,233 @@
+"""Thin ctypes binding of libratel.so -- same names as include/ratel.h.
+
+Argument marshalling only: every step of the optimizer path runs in the CUDA
+library.  There is no fallback: if libratel.so is missing or fails to load,
+importing this module raises ImportError.
+
+Errors: a non-zero status becomes ``RatelError(code, message)`` carrying the
+C code (RATEL_EINVAL, RATEL_ESTATE, ...) and ratel_last_error()'s text.
+Pointers are passed as integers (``tensor.data_ptr()``); CUDA streams as
+integers (``torch.cuda.Stream.cuda_stream``) or None.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libratel.so")
+
+RATEL_OK = 0
+RATEL_EINVAL = -1
+RATEL_ESTATE = -2
+RATEL_ECUDA = -3
+RATEL_ENCCL = -4
+RATEL_ENOMEM = -5
+RATEL_ENONFINITE = -6
+
+RATEL_DEVICE = 0
+RATEL_PINNED_HOST = 1
+RATEL_ADAMW = 0
+RATEL_ADAM_L2 = 1
+RATEL_STAGING_PIPELINED = 0
+RATEL_STAGING_SERIALIZED = 1
+RATEL_MAX_BLOCKS = 4096
+RATEL_MAX_RANGES_PER_BLOCK = 32
+
+_NAMES = {0: "RATEL_OK", -1: "RATEL_EINVAL", -2: "RATEL_ESTATE", -3: "RATEL_ECUDA",
+          -4: "RATEL_ENCCL", -5: "RATEL_ENOMEM", -6: "RATEL_ENONFINITE"}
+
+
+class RatelError(RuntimeError):
+    def __init__(self, code: int, msg: str):
+        super().__init__(f"{_NAMES.get(code, code)}: {msg}")
+        self.code = code
+
+
+class ratel_config(ctypes.Structure):
+    _fields_ = [
+        ("mode", ctypes.c_int),
+        ("max_grad_norm", ctypes.c_double),
+        ("pipeline_depth", ctypes.c_int),
+        ("staging", ctypes.c_int),
+        ("tile_elems", ctypes.c_uint64),
+        ("max_ctas", ctypes.c_int),
+        ("timing", ctypes.c_int),
+    ]
+
+
+class ratel_range(ctypes.Structure):
+    _fields_ = [
+        ("param_bf16", ctypes.c_void_p),
+        ("grad_bf16", ctypes.c_void_p),
+        ("grad_is_rank_slice", ctypes.c_int),
+        ("master", ctypes.c_void_p),
+        ("exp_avg", ctypes.c_void_p),
+        ("exp_avg_sq", ctypes.c_void_p),
+        ("numel", ctypes.c_uint64),
+        ("apply_weight_decay", ctypes.c_int),
+    ]
+
+
+def _load():
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(f"{_LIB_PATH} is missing: build it with "
+                          "`python -c 'import __graft_entry__ as g; g.build()'` (no CPU fallback exists)")
+    lib = ctypes.CDLL(_LIB_PATH)
+    P, I, U64, D = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint64, ctypes.c_double
+    sig = {
+        "ratel_default_config": (None, [ctypes.POINTER(ratel_config)]),
+        "ratel_get_nccl_unique_id": (I, [P]),
+        "ratel_init": (I, [I, I, I, P, ctypes.POINTER(ratel_config)]),
+        "ratel_register_block": (I, [I, ctypes.POINTER(ratel_range), I, I]),
+        "ratel_adam_step": (I, [D, D, D, D, D, ctypes.c_int64]),
+        "ratel_offload_grad_chunk": (I, [I, P]),
+        "ratel_sync": (I, [P]),
+        "ratel_finalize": (I, []),
+        "ratel_last_error": (ctypes.c_char_p, []),
+        "ratel_padded_numel": (U64, [U64, I]),
+        "ratel_rank_slice": (I, [U64, I, I, ctypes.POINTER(U64), ctypes.POINTER(U64)]),
+        "ratel_optimizer_stream": (P, []),
+        "ratel_get_grad_sumsq": (I, [ctypes.POINTER(D)]),
+        "ratel_kernel_timing": (I, [ctypes.POINTER(D), ctypes.POINTER(ctypes.c_int64), I]),
+        "ratel_launch_count": (ctypes.c_int64, []),
+        "ratel_gen_stream_key": (U64, [U64, U64, U64, U64]),
+        "ratel_gen_theta0": (I, [P, U64, U64, U64, P]),
+        "ratel_gen_grad16": (I, [P, U64, U64, U64, P]),
+        "ratel_test_bf16_rne": (I, [P, P, U64, P]),
+        "ratel_test_fill_f32": (I, [P, U64, ctypes.c_float, P]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    return lib
+
+
+_lib = _load()
+LIB_PATH = _LIB_PATH
+
+
+def lib():
+    return _lib
+
+
+def _check(rc: int) -> None:
+    if rc != RATEL_OK:
+        raise RatelError(rc, (_lib.ratel_last_error() or b"").decode(errors="replace"))
+
+
+def _stream(s):
+    if s is None:
+        return None
+    if hasattr(s, "cuda_stream"):
+        return s.cuda_stream
+    return int(s)
+
+
+# --------------------------------------------------------------------- ABI
+def ratel_default_config() -> ratel_config:
+    c = ratel_config()
+    _lib.ratel_default_config(ctypes.byref(c))
+    return c
+
+
+def ratel_get_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(_lib.ratel_get_nccl_unique_id(buf))
+    return buf.raw
+
+
+def ratel_init(device: int, rank: int = 0, world_size: int = 1, nccl_unique_id: bytes | None = None,
+               cfg: ratel_config | None = None) -> None:
+    uid = None
+    if nccl_unique_id is not None:
+        assert len(nccl_unique_id) == 128
+        uid = ctypes.create_string_buffer(bytes(nccl_unique_id), 128)
+    _check(_lib.ratel_init(device, rank, world_size, uid, ctypes.byref(cfg) if cfg is not None else None))
+
+
+def ratel_register_block(block_id: int, ranges, residency: int = RATEL_DEVICE) -> None:
+    arr = (ratel_range * len(ranges))(*ranges)
+    _check(_lib.ratel_register_block(block_id, arr, len(ranges), residency))
+
+
+def ratel_adam_step(lr: float, beta1: float, beta2: float, eps: float, weight_decay: float, step: int) -> None:
+    _check(_lib.ratel_adam_step(lr, beta1, beta2, eps, weight_decay, step))
+
+
+def ratel_offload_grad_chunk(block_id: int, stream=None) -> None:
+    _check(_lib.ratel_offload_grad_chunk(block_id, _stream(stream)))
+
+
+def ratel_sync(stream=None) -> None:
+    _check(_lib.ratel_sync(_stream(stream)))
+
+
+def ratel_finalize() -> None:
+    _check(_lib.ratel_finalize())
+
+
+def ratel_last_error() -> str:
+    return (_lib.ratel_last_error() or b"").decode(errors="replace")
+
+
+def ratel_padded_numel(numel: int, world_size: int) -> int:
+    return int(_lib.ratel_padded_numel(numel, world_size))
+
+
+def ratel_rank_slice(numel: int, world_size: int, rank: int) -> tuple[int, int]:
+    b, e = ctypes.c_uint64(), ctypes.c_uint64()
+    _check(_lib.ratel_rank_slice(numel, world_size, rank, ctypes.byref(b), ctypes.byref(e)))
+    return int(b.value), int(e.value)
+
+
+def ratel_optimizer_stream() -> int | None:
+    return _lib.ratel_optimizer_stream()
+
+
+def ratel_get_grad_sumsq() -> float:
+    out = ctypes.c_double()
+    _check(_lib.ratel_get_grad_sumsq(ctypes.byref(out)))
+    return out.value
+
+
+def ratel_kernel_timing(reset: bool = False) -> tuple[float, int]:
+    ms, n = ctypes.c_double(), ctypes.c_int64()
+    _check(_lib.ratel_kernel_timing(ctypes.byref(ms), ctypes.byref(n), int(reset)))
+    return ms.value, n.value
+
+
+def ratel_launch_count() -> int:
+    return int(_lib.ratel_launch_count())
+
+
+# -------------------------------------------------- include/ratel_gen.h
+def ratel_gen_stream_key(seed: int, tag: int, step: int, block: int) -> int:
+    return int(_lib.ratel_gen_stream_key(seed, tag, step, block))
+
+
+def ratel_gen_theta0(dst_ptr: int, n: int, start: int, key: int, stream=None) -> None:
+    _check(_lib.ratel_gen_theta0(dst_ptr, n, start, key, _stream(stream)))
+
+
+def ratel_gen_grad16(dst_ptr: int, n: int, start: int, key: int, stream=None) -> None:
+    _check(_lib.ratel_gen_grad16(dst_ptr, n, start, key, _stream(stream)))
+
+
+def ratel_test_bf16_rne(in_ptr: int, out_ptr: int, n: int, stream=None) -> None:
+    _check(_lib.ratel_test_bf16_rne(in_ptr, out_ptr, n, _stream(stream)))
+
+
+def ratel_test_fill_f32(dst_ptr: int, n: int, value: float, stream=None) -> None:
+    _check(_lib.ratel_test_fill_f32(dst_ptr, n, value, _stream(stream)))
+
+
+def make_range(param, grad, master, exp_avg, exp_avg_sq, numel: int, apply_weight_decay: int = 1,
+               grad_is_rank_slice: int = 0) -> ratel_range:
+    """Build a ratel_range from tensors (or raw integer pointers)."""
+    def p(x):
+        if x is None:
+            return None
+        return x.data_ptr() if hasattr(x, "data_ptr") else int(x)
+    return ratel_range(p(param), p(grad), grad_is_rank_slice, p(master), p(exp_avg), p(exp_avg_sq),
+                       numel, apply_weight_decay)

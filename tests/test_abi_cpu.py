@@ -1,0 +1,121 @@
+"""C-ABI library checks that need no GPU: it loads, exports every symbol the
+headers declare, its host-only functions (partition, generator keys) are
+right, and every stateful call fails cleanly without a device."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+import synth
+import paper_conf_icde_liaosyxcyww25_b200 as R
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def declared_functions():
+    names = []
+    for h in ("ratel.h", "ratel_gen.h"):
+        src = open(os.path.join(ROOT, "include", h)).read()
+        src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+        names += re.findall(r"^[A-Za-z_][\w\s\*]*?\b(ratel_\w+)\s*\(", src, flags=re.M)
+    return sorted(set(names))
+
+
+def test_exports_every_declared_symbol():
+    names = declared_functions()
+    assert len(names) >= 20, names
+    lib = ctypes.CDLL(R.LIB_PATH)
+    missing = [n for n in names if not hasattr(lib, n)]
+    assert not missing, missing
+
+
+def test_built_for_sm100a_only():
+    out = os.popen(f"cuobjdump -lelf {R.LIB_PATH} 2>/dev/null").read()
+    if not out:
+        pytest.skip("cuobjdump unavailable")
+    archs = set(re.findall(r"sm_(\d+a?)", out))
+    assert archs == {"100a"}, archs
+
+
+def test_stateful_calls_without_init_are_estate():
+    for f in (lambda: R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 0.0, 1),
+              lambda: R.ratel_offload_grad_chunk(0, None),
+              lambda: R.ratel_sync(None),
+              lambda: R.ratel_finalize(),
+              lambda: R.ratel_get_grad_sumsq()):
+        with pytest.raises(R.RatelError) as e:
+            f()
+        assert e.value.code == R.RATEL_ESTATE
+    assert R.ratel_optimizer_stream() is None
+    assert R.ratel_launch_count() == 0
+
+
+def test_init_without_gpu_fails_cleanly():
+    with pytest.raises(R.RatelError) as e:
+        R.ratel_init(0)
+    assert e.value.code in (R.RATEL_ECUDA, R.RATEL_EINVAL)
+    assert "device" in R.ratel_last_error() or "CUDA" in R.ratel_last_error()
+    # bad arguments are rejected before touching CUDA
+    with pytest.raises(R.RatelError) as e:
+        R.ratel_init(0, 2, 2, None)
+    assert e.value.code == R.RATEL_EINVAL
+    with pytest.raises(R.RatelError) as e:
+        R.ratel_init(0, 1, 2, None)  # world > 1 needs a unique id
+    assert e.value.code == R.RATEL_EINVAL
+    cfg = R.ratel_default_config()
+    cfg.pipeline_depth = 4
+    with pytest.raises(R.RatelError) as e:
+        R.ratel_init(0, 0, 1, None, cfg)
+    assert e.value.code == R.RATEL_EINVAL
+
+
+def test_default_config():
+    c = R.ratel_default_config()
+    assert (c.mode, c.max_grad_norm, c.pipeline_depth, c.staging, c.tile_elems, c.max_ctas, c.timing) == \
+        (R.RATEL_ADAMW, 0.0, 3, R.RATEL_STAGING_PIPELINED, 1 << 24, 0, 0)
+
+
+@pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
+def test_partition_covers_range_exactly(world):
+    """Slices of every rank tile [0, n) in order, disjointly; each slice
+    starts at a multiple of 8 elements (16-byte aligned for bf16 and fp32);
+    all ranks own ceil-equal shares."""
+    rng = np.random.default_rng(world)
+    ns = [1, 7, 8, 9, 63, 64, 65, 8 * world, 8 * world + 1, 789_760, 314_639_360, 1_812_099_072]
+    ns += [int(x) for x in rng.integers(1, 10 ** 7, 50)]
+    for n in ns:
+        cap = R.ratel_padded_numel(n, world)
+        assert cap >= n and cap % (8 * world) == 0 and cap - n < 8 * world
+        s = cap // world
+        prev = 0
+        for r in range(world):
+            b, e = R.ratel_rank_slice(n, world, r)
+            assert b == min(n, r * s) and e == min(n, b + s)
+            assert b == prev or b == n
+            assert b % 8 == 0 or b == n
+            prev = e
+        assert prev == n
+
+
+def test_rank_slice_rejects_bad_args():
+    with pytest.raises(R.RatelError):
+        R.ratel_rank_slice(10, 2, 2)
+    with pytest.raises(R.RatelError):
+        R.ratel_rank_slice(10, 0, 0)
+    assert R.ratel_padded_numel(10, 0) == 0
+
+
+def test_generator_keys_match_synth():
+    for args in [(synth.SEED, 1, 0, 0), (synth.SEED, 2, 7, 40), (0, 0, 0, 0), (2 ** 64 - 1, 5, 2 ** 40, 3)]:
+        assert R.ratel_gen_stream_key(*args) == synth.stream_key(*args)
+
+
+def test_struct_layouts_match_header():
+    # ratel_config: int, double, int, int, uint64, int, int -> 40 bytes
+    assert ctypes.sizeof(R.ratel_config) == 40
+    assert R.ratel_config.tile_elems.offset == 24
+    # ratel_range: 2 ptrs, int, 3 ptrs, uint64, int -> 64 bytes
+    assert ctypes.sizeof(R.ratel_range) == 64
+    assert R.ratel_range.master.offset == 24 and R.ratel_range.numel.offset == 48

@@ -1,0 +1,334 @@
+"""GPU parity: the CUDA path through the C ABI vs the CPU oracle.
+
+Bounds: DESIGN.md R13 (tests/tolerance.py) at tol 1e-5 -- BASELINE.json's
+"max relative error 1e-5" and "bf16 within 1 ulp" read against the scale the
+oracle tracks.  Self-consistency claims (R16) are bitwise.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+import paper_conf_icde_liaosyxcyww25_b200 as R
+from tests.harness import HP, GpuBlock, ratel_lib, torch_to_u16, u16_to_torch
+from tests.tolerance import check_range
+
+pytestmark = pytest.mark.gpu
+
+# C1 (BASELINE.json configs[0]): one GPT block, h = 256 -> 12h^2 + 13h params,
+# the 12 tensors of SURVEY §8(d): ln1 w/b, qkv W/b, proj W/b, ln2 w/b, fc1 W/b, fc2 W/b.
+H = 256
+C1_SIZES = [H, H, 3 * H * H, 3 * H, H * H, H, H, H, 4 * H * H, 4 * H, 4 * H * H, H]
+C1_WD = [0, 0, 1, 0, 1, 0, 0, 0, 1, 0, 1, 0]
+assert sum(C1_SIZES) == 789_760
+
+
+def oracle_step(blocks, step, grads, mode=oracle.ADAMW, max_norm=0.0, **hp):
+    h = dict(HP, **hp)
+    rs, gs = [], []
+    for b in blocks:
+        rs += b.oracle
+        gs += grads[b.id]
+    return oracle.adam_step(rs, gs, oracle.hparams(step=step, mode=mode, **h), max_grad_norm=max_norm)
+
+
+def run(blocks, steps, mode=oracle.ADAMW, max_norm=0.0, order="decreasing", arm="before",
+        check_every=True, tol=1e-5, hp_sched=None, **cfg_kw):
+    """Drive `steps` optimizer steps through the ABI and the oracle; check."""
+    dev = blocks[0].dev
+    reports = []
+    with ratel_lib(mode=mode, max_grad_norm=max_norm, **cfg_kw):
+        for b in blocks:
+            b.register()
+        bwd = torch.cuda.Stream()
+        rng = np.random.default_rng(7)
+        for t in range(1, steps + 1):
+            h = dict(HP)
+            if hp_sched:
+                h.update(hp_sched(t))
+            grads = {}
+            for b in blocks:
+                grads[b.id] = b.load_grads(t)
+            torch.cuda.synchronize()
+            ids = [b.id for b in blocks]
+            if order == "decreasing":
+                ids = sorted(ids, reverse=True)
+            elif order == "random":
+                ids = list(rng.permutation(ids))
+            if arm == "before":
+                R.ratel_adam_step(h["lr"], h["beta1"], h["beta2"], h["eps"], h["weight_decay"], t)
+            for i in ids:
+                R.ratel_offload_grad_chunk(int(i), bwd)
+            if arm == "after":
+                R.ratel_adam_step(h["lr"], h["beta1"], h["beta2"], h["eps"], h["weight_decay"], t)
+            R.ratel_sync(None)
+            S, coef = oracle_step(blocks, t, grads, mode=mode, max_norm=max_norm, **h)
+            if max_norm > 0:
+                got = R.ratel_get_grad_sumsq()
+                n_all = sum(sum(b.sizes) for b in blocks)  # positive terms: |err| <= n u S
+                assert abs(got - S) <= n_all * 2.0 ** -53 * S, (got, S)
+            if check_every or t == steps:
+                for b in blocks:
+                    for i in range(len(b.sizes)):
+                        reports.append(check_range(b.gpu_state(i), b.oracle[i], tol=tol,
+                                                   own_rne=oracle.bf16_rne,
+                                                   what=f"step {t} block {b.id} range {i}"))
+    return reports
+
+
+def snapshot(blocks):
+    return [[b.gpu_state(i) for i in range(len(b.sizes))] for b in blocks]
+
+
+def assert_bitwise(sa, sb):
+    for xa, xb in zip(sa, sb):
+        for ra, rb in zip(xa, xb):
+            for k in ("p32", "m32", "v32", "p16"):
+                assert np.array_equal(ra[k].view(np.uint32) if ra[k].dtype == np.float32 else ra[k],
+                                      rb[k].view(np.uint32) if rb[k].dtype == np.float32 else rb[k]), k
+
+
+# ------------------------------------------------------------------ C1 parity
+def test_c1_flat_range_10_steps(cuda_dev):
+    b = GpuBlock(0, [sum(C1_SIZES)], cuda_dev)
+    reps = run([b], 10)
+    worst = max(r["theta_scaled"] for r in reps)
+    assert worst < 1e-5
+    print("C1 flat worst scaled errors:", {k: max(r[k] for r in reps)
+                                           for k in ("theta_scaled", "m_scaled", "v_rel", "p16_ulps_at_scale")})
+
+
+def test_c1_twelve_ranges_wd_exempt(cuda_dev):
+    b = GpuBlock(0, C1_SIZES, cuda_dev, wd_flags=C1_WD)
+    run([b], 10)
+
+
+def test_c1_adam_l2_mode(cuda_dev):
+    b = GpuBlock(0, C1_SIZES, cuda_dev, wd_flags=C1_WD)
+    run([b], 10, mode=oracle.ADAM_L2)
+
+
+def test_lr_schedule_flows_per_step(cuda_dev):
+    b = GpuBlock(3, [100_003], cuda_dev)
+    run([b], 6, hp_sched=lambda t: dict(lr=1e-3 * (0.5 ** t), weight_decay=0.1 * t))
+
+
+@pytest.mark.parametrize("max_norm", [1e-3, 1e6])
+def test_clip_global_norm(cuda_dev, max_norm):
+    blocks = [GpuBlock(i, [50_000 + 13 * i, 777], cuda_dev) for i in range(3)]
+    run(blocks, 5, max_norm=max_norm)
+
+
+def test_ragged_sizes_many_blocks(cuda_dev):
+    sizes = [[1], [7], [8], [9], [15, 17], [1023], [1_000_003], [4096 * 3 + 5, 1]]
+    blocks = [GpuBlock(i, s, cuda_dev) for i, s in enumerate(sizes)]
+    run(blocks, 4, order="random")
+
+
+def test_special_values_propagate(cuda_dev):
+    """Non-finite grads propagate (torch default, R8); eps, zeros handled."""
+    b = GpuBlock(0, [64], cuda_dev)
+    with ratel_lib():
+        b.register()
+        g = b.grads_np(1)[0].copy()
+        g[:6] = [0x7F80, 0xFF80, 0x7FC0, 0x0000, 0x8000, 0x0001]  # +inf -inf nan +0 -0 denormal
+        b.g16[0][:64].copy_(u16_to_torch(g, cuda_dev))
+        torch.cuda.synchronize()
+        R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, 1)
+        R.ratel_offload_grad_chunk(0, None)
+        R.ratel_sync(None)
+        oracle.adam_range(b.oracle[0], g, oracle.hparams(step=1))
+        check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne)
+
+
+# ------------------------------------------------ self-consistency (R16)
+def _fresh(sizes_list, dev, **kw):
+    return [GpuBlock(i, s, dev, **kw) for i, s in enumerate(sizes_list)]
+
+
+SIZES = [[300_001], [65_536 + 24], [4_000, 12, 999]]
+
+
+def test_bitwise_handoff_order_and_deferred(cuda_dev):
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 3, order="decreasing", arm="before", check_every=False)
+    b = _fresh(SIZES, cuda_dev)
+    run(b, 3, order="random", arm="before", check_every=False)
+    c = _fresh(SIZES, cuda_dev)
+    run(c, 3, order="decreasing", arm="after", check_every=False)  # "Ratel+ZeRO" deferred
+    sa = snapshot(a)
+    assert_bitwise(sa, snapshot(b))
+    assert_bitwise(sa, snapshot(c))
+
+
+@pytest.mark.parametrize("depth,staging,tile", [(2, 0, 4096), (3, 0, 65_536), (3, 1, 8192), (2, 0, 1 << 24)])
+def test_pinned_host_bitwise_equals_device(cuda_dev, depth, staging, tile):
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 3, check_every=False)
+    b = _fresh(SIZES, cuda_dev, pinned=True)
+    run(b, 3, check_every=False, pipeline_depth=depth, staging=staging, tile_elems=tile)
+    assert_bitwise(snapshot(a), snapshot(b))
+
+
+def test_max_ctas_cap_bitwise(cuda_dev):
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 2, check_every=False)
+    b = _fresh(SIZES, cuda_dev)
+    run(b, 2, check_every=False, max_ctas=3)
+    assert_bitwise(snapshot(a), snapshot(b))
+
+
+def test_overlapped_with_backward_stream(cuda_dev):
+    """Grads are produced on a side stream right before each hand-off (the
+    AGO pattern); a busy GEMM keeps that stream occupied so K1 must wait on
+    the event, not on host order."""
+    blocks = _fresh([[200_000], [150_000], [99_999]], cuda_dev)
+    with ratel_lib():
+        for b in blocks:
+            b.register()
+        bwd = torch.cuda.Stream()
+        x = torch.randn(4096, 4096, device=cuda_dev, dtype=torch.bfloat16)
+        for t in (1, 2, 3):
+            grads = {b.id: b.grads_np(t) for b in blocks}
+            host = {b.id: [u16_to_torch(g, "cpu").pin_memory() for g in grads[b.id]] for b in blocks}
+            torch.cuda.synchronize()
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            with torch.cuda.stream(bwd):
+                for b in sorted(blocks, key=lambda b: -b.id):
+                    for _ in range(4):
+                        x = (x @ x).clamp_(-1, 1)          # "backward" work
+                    for i, hg in enumerate(host[b.id]):
+                        b.g16[i][:hg.numel()].copy_(hg, non_blocking=True)
+                    for gt in b.g16:
+                        gt.record_stream(torch.cuda.ExternalStream(R.ratel_optimizer_stream()))
+                    R.ratel_offload_grad_chunk(b.id, bwd)
+            R.ratel_sync(torch.cuda.current_stream())
+            torch.cuda.synchronize()
+            oracle_step(blocks, t, grads)
+            for b in blocks:
+                check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne)
+
+
+def test_no_staleness_after_stream_sync(cuda_dev):
+    """ratel_sync(stream): work queued on `stream` afterwards sees the updated
+    P16, which equals bf16_rne(P32) bit for bit (footnote 4)."""
+    b = GpuBlock(0, [1 << 20], cuda_dev)
+    with ratel_lib():
+        b.register()
+        s = torch.cuda.Stream()
+        for t in (1, 2):
+            b.load_grads(t)
+            torch.cuda.synchronize()
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            R.ratel_offload_grad_chunk(0, None)
+            R.ratel_sync(s)
+            with torch.cuda.stream(s):
+                snap = b.p16[0].clone()
+                want = b.master[0].to(torch.bfloat16)  # torch's RNE cast, independent of K1
+            s.synchronize()
+            assert torch.equal(snap.view(torch.int16), want.view(torch.int16))
+
+
+# --------------------------------------------------------- protocol errors
+def test_protocol_errors(cuda_dev):
+    b = GpuBlock(0, [1000], cuda_dev)
+    c = GpuBlock(1, [1000], cuda_dev)
+    with ratel_lib():
+        b.register()
+        c.register()
+        with pytest.raises(R.RatelError) as e:
+            b.register()
+        assert e.value.code == R.RATEL_EINVAL
+        R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 0.0, 1)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 0.0, 2)  # already armed
+        assert e.value.code == R.RATEL_ESTATE
+        R.ratel_offload_grad_chunk(0, None)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_offload_grad_chunk(0, None)
+        assert e.value.code == R.RATEL_ESTATE
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_sync(None)  # block 1 missing
+        assert e.value.code == R.RATEL_ESTATE
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_offload_grad_chunk(7, None)
+        assert e.value.code == R.RATEL_ESTATE
+        R.ratel_offload_grad_chunk(1, None)
+        R.ratel_sync(None)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 0.0, 1)  # step must increase
+        assert e.value.code == R.RATEL_ESTATE
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_adam_step(1e-3, 1.0, 0.999, 1e-8, 0.0, 5)
+        assert e.value.code == R.RATEL_EINVAL
+        # pointer validation: pageable host memory, misalignment, wrong kind
+        pageable = torch.zeros(1000, dtype=torch.float32)
+        bad = R.make_range(b.p16[0], b.g16[0], pageable, pageable, pageable, 1000)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_register_block(5, [bad], R.RATEL_PINNED_HOST)
+        assert e.value.code == R.RATEL_EINVAL
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_register_block(5, [bad], R.RATEL_DEVICE)
+        assert e.value.code == R.RATEL_EINVAL
+        mis = R.make_range(b.p16[0].data_ptr() + 2, b.g16[0], b.master[0], b.m[0], b.v[0], 100)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_register_block(5, [mis], R.RATEL_DEVICE)
+        assert e.value.code == R.RATEL_EINVAL
+        # still healthy (EINVAL/ESTATE are not sticky)
+        R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 0.0, 9)
+        R.ratel_offload_grad_chunk(1, None)
+        R.ratel_offload_grad_chunk(0, None)
+        R.ratel_sync(None)
+    with pytest.raises(R.RatelError) as e:
+        R.ratel_sync(None)
+    assert e.value.code == R.RATEL_ESTATE
+
+
+def test_nonfinite_norm_reported(cuda_dev):
+    b = GpuBlock(0, [4096], cuda_dev)
+    with ratel_lib(max_grad_norm=1.0):
+        b.register()
+        g = b.grads_np(1)[0].copy()
+        g[5] = 0x7FC0
+        b.g16[0][:4096].copy_(u16_to_torch(g, cuda_dev))
+        torch.cuda.synchronize()
+        R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, 1)
+        R.ratel_offload_grad_chunk(0, None)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_sync(None)
+        assert e.value.code == R.RATEL_ENONFINITE
+        assert np.isnan(b.gpu_state(0)["p32"]).all()  # NaN coef propagates like torch
+
+
+# -------------------------------------------------------- conversions / inputs
+def test_gpu_bf16_rne_exhaustive(cuda_dev):
+    """The device P16 conversion == the oracle's RNE for all 2^32 fp32 patterns
+    (NaN: both NaN)."""
+    chunk = 1 << 28
+    out = torch.empty(chunk, dtype=torch.int16, device=cuda_dev)
+    for start in range(0, 1 << 32, chunk):
+        u = torch.arange(start, start + chunk, dtype=torch.int64, device=cuda_dev).to(torch.int32)
+        x = u.view(torch.float32)
+        R.ratel_test_bf16_rne(x.data_ptr(), out.data_ptr(), chunk)
+        got = out.cpu().numpy().view(np.uint16)
+        xs = x.cpu().numpy()
+        ref = oracle.bf16_rne(xs)
+        isn = np.isnan(xs)
+        assert np.array_equal(got[~isn], ref[~isn]), start
+        assert np.all((got[isn] & 0x7FFF) > 0x7F80)
+
+
+def test_device_generator_matches_synth(cuda_dev):
+    n, start = 3_000_017, 123_456_789
+    for blk, step in ((0, 1), (5, 9)):
+        kg = R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, step, blk)
+        kt = R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, blk)
+        assert kg == synth.stream_key(synth.SEED, synth.TAG_GRAD, step, blk)
+        g = torch.empty(n, dtype=torch.int16, device=cuda_dev)
+        th = torch.empty(n, dtype=torch.float32, device=cuda_dev)
+        R.ratel_gen_grad16(g.data_ptr(), n, start, kg)
+        R.ratel_gen_theta0(th.data_ptr(), n, start, kt)
+        assert np.array_equal(g.cpu().numpy().view(np.uint16), synth.grad16(n, step, blk, start=start))
+        assert np.array_equal(th.cpu().numpy().view(np.uint32),
+                              synth.theta0(n, blk, start=start).view(np.uint32))
