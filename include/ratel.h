@@ -43,7 +43,8 @@
  * e.g. torch) and must stay valid and unmoved until ratel_finalize.  Between
  * a block's hand-off and ratel_sync the caller must not touch that block's
  * master/exp_avg/exp_avg_sq/param nor overwrite its grad (in torch:
- * grad.record_stream(ratel_optimizer_stream())).  The library owns only what
+ * grad.record_stream(ratel_optimizer_stream()); such tensors must be
+ * released before ratel_finalize destroys that stream).  The library owns only what
  * it creates: streams, events, device tiles, reduction buffers, NCCL comm.
  *
  * Errors: every int-returning call returns RATEL_OK (0) or a negative code.

@@ -49,11 +49,14 @@ def stale() -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not stale():
+def build(force: bool = False, verbose: bool = False, out: str | None = None, defines=()) -> str:
+    """Compile libratel.so; `out`/`defines` build a variant elsewhere (tools)."""
+    target = out or LIB
+    if out is None and not force and not stale():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = target + f".tmp{os.getpid()}"
     cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2",
+           *[f"-D{d}" for d in defines],
            "-Xptxas", "-v" if verbose else "-O3", "-shared", "-o", tmp,
            "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(),
            *[os.path.join(CSRC, f) for f in SOURCES], "-ldl"]
@@ -63,8 +66,8 @@ def build(force: bool = False, verbose: bool = False) -> str:
         raise RuntimeError("nvcc failed building libratel.so")
     if verbose:
         sys.stderr.write(r.stderr)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -37,7 +37,8 @@ struct AdamScalars {
   float inv_sqrt_bc2;             // 1 / sqrt(1 - b2^t)
   float eps;
   float decay;                    // 1 - lr*wd      (AdamW)
-  float wd;                       // wd             (Adam-L2)
+  float wd;                       // wd             (unused; kept for layout clarity)
+  double wd_d;                    // wd in double   (Adam-L2, see adam_update)
 };
 
 // One rank-slice (or one staged tile) of a parameter range.
@@ -68,10 +69,19 @@ struct SumsqParams {
   double* partials;  // one slot per CTA
 };
 
+#ifndef RATEL_K1_FASTMATH
+#define RATEL_K1_FASTMATH 1
+#endif
+
 // The per-element update.  Explicit-rounding intrinsics fix the operation
 // sequence (no contraction freedom):
 //   AdamW:   theta = theta*decay            (wd_on)
-//   Adam-L2: g     = fma(wd, theta, g)      (wd_on)
+//   Adam-L2: g     = fp32(fma(wd, theta, g) in fp64)   (wd_on)
+// The L2 term is formed in double: g and wd*theta cancel when the gradient
+// balances the decay, and fp32(wd) alone (rel. error 2e-8) would then move
+// g' by more than its own ulp and the update by >1e-5 of its scale near
+// |g'| ~ eps (measured on B200; R3).  One DFMA per element is far
+// inside the ALU budget of this HBM-bound kernel.
 //   m     = fma(b1, m, (1-b1)*g)
 //   v     = fma(b2, v, (1-b2)*(g*g))        g*g is exact for a bf16 g
 //   denom = fma(sqrt(v), 1/sqrt(bc2), eps)  == sqrt(v/bc2) + eps
@@ -80,65 +90,122 @@ template <int MODE>
 __device__ __forceinline__ void adam_update(float g, float& th, float& m, float& v,
                                             const AdamScalars& s, bool wd_on) {
   if (MODE == RATEL_ADAM_L2) {
-    if (wd_on) g = __fmaf_rn(s.wd, th, g);
+    if (wd_on) g = __double2float_rn(__fma_rn(s.wd_d, static_cast<double>(th), static_cast<double>(g)));
   } else {
     if (wd_on) th = __fmul_rn(th, s.decay);
   }
   m = __fmaf_rn(s.beta1, m, __fmul_rn(s.one_minus_beta1, g));
   v = __fmaf_rn(s.beta2, v, __fmul_rn(s.one_minus_beta2, __fmul_rn(g, g)));
+#if RATEL_K1_FASTMATH
+  float sq, r;
+  asm("sqrt.approx.f32 %0, %1;" : "=f"(sq) : "f"(v));
+  const float denom = __fmaf_rn(sq, s.inv_sqrt_bc2, s.eps);
+  asm("rcp.approx.f32 %0, %1;" : "=f"(r) : "f"(denom));
+  th = __fmaf_rn(s.neg_step_size, __fmul_rn(m, r), th);
+#else
   const float denom = __fmaf_rn(__fsqrt_rn(v), s.inv_sqrt_bc2, s.eps);
   th = __fmaf_rn(s.neg_step_size, __fdiv_rn(m, denom), th);
+#endif
 }
 
-// 8 consecutive elements: 1x16 B of g, 2x16 B each of theta, m, v.
+// ---- K1 memory operations --------------------------------------------------
+// Build-time variants (tools/k1_sweep.py measures them on the B200):
+//   RATEL_K1_LDST 0: 2 x 128-bit ld/st.global.cs per fp32 octet
+//                 1: 256-bit ld/st (sm_100) with L1::no_allocate + L2::evict_first
+//                 2: 256-bit ld/st, no cache hints
+//   RATEL_K1_UNROLL  octets in flight per thread per loop trip
+//   RATEL_K1_MINB    __launch_bounds__ min CTAs/SM (register budget)
+#ifndef RATEL_K1_LDST
+#define RATEL_K1_LDST 2
+#endif
+#ifndef RATEL_K1_UNROLL
+#define RATEL_K1_UNROLL 2
+#endif
+#ifndef RATEL_K1_MINB
+#define RATEL_K1_MINB 2
+#endif
+
+__device__ __forceinline__ void ld_f8(const float* p, float (&r)[8]) {
+#if RATEL_K1_LDST == 0
+  const float4 a = __ldcs(reinterpret_cast<const float4*>(p));
+  const float4 b = __ldcs(reinterpret_cast<const float4*>(p) + 1);
+  r[0] = a.x; r[1] = a.y; r[2] = a.z; r[3] = a.w; r[4] = b.x; r[5] = b.y; r[6] = b.z; r[7] = b.w;
+#elif RATEL_K1_LDST == 1
+  asm volatile("ld.global.L1::no_allocate.L2::evict_first.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]), "=f"(r[7])
+               : "l"(p));
+#else
+  asm volatile("ld.global.v8.f32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=f"(r[0]), "=f"(r[1]), "=f"(r[2]), "=f"(r[3]), "=f"(r[4]), "=f"(r[5]), "=f"(r[6]), "=f"(r[7])
+               : "l"(p));
+#endif
+}
+
+__device__ __forceinline__ void st_f8(float* p, const float (&r)[8]) {
+#if RATEL_K1_LDST == 0
+  __stcs(reinterpret_cast<float4*>(p), make_float4(r[0], r[1], r[2], r[3]));
+  __stcs(reinterpret_cast<float4*>(p) + 1, make_float4(r[4], r[5], r[6], r[7]));
+#elif RATEL_K1_LDST == 1
+  asm volatile("st.global.L1::no_allocate.L2::evict_first.v8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+               :: "l"(p), "f"(r[0]), "f"(r[1]), "f"(r[2]), "f"(r[3]), "f"(r[4]), "f"(r[5]), "f"(r[6]), "f"(r[7])
+               : "memory");
+#else
+  asm volatile("st.global.v8.f32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};"
+               :: "l"(p), "f"(r[0]), "f"(r[1]), "f"(r[2]), "f"(r[3]), "f"(r[4]), "f"(r[5]), "f"(r[6]), "f"(r[7])
+               : "memory");
+#endif
+}
+
+__device__ __forceinline__ uint4 ld_g8(const uint16_t* p) {
+#if RATEL_K1_LDST != 2  // (.L2::evict_first exists only for 256-bit accesses)
+  return __ldcs(reinterpret_cast<const uint4*>(p));
+#else
+  return *reinterpret_cast<const uint4*>(p);
+#endif
+}
+
+__device__ __forceinline__ void st_p8(uint16_t* p, uint4 v) {
+#if RATEL_K1_LDST == 2
+  *reinterpret_cast<uint4*>(p) = v;
+#else
+  __stcs(reinterpret_cast<uint4*>(p), v);
+#endif
+}
+
+// 8 consecutive elements: 16 B of g, 32 B each of theta, m, v.
 struct Frag8 {
   uint4 g;
-  float4 t0, t1, m0, m1, v0, v1;
+  float t[8], m[8], v[8];
 };
 
 __device__ __forceinline__ void load8(Frag8& f, const RangeDesc& R, uint64_t i) {
-  f.g = __ldcs(reinterpret_cast<const uint4*>(R.g) + i);
-  const float4* th = reinterpret_cast<const float4*>(R.th) + 2 * i;
-  const float4* m = reinterpret_cast<const float4*>(R.m) + 2 * i;
-  const float4* v = reinterpret_cast<const float4*>(R.v) + 2 * i;
-  f.t0 = __ldcs(th);
-  f.t1 = __ldcs(th + 1);
-  f.m0 = __ldcs(m);
-  f.m1 = __ldcs(m + 1);
-  f.v0 = __ldcs(v);
-  f.v1 = __ldcs(v + 1);
+  f.g = ld_g8(R.g + 8 * i);
+  ld_f8(R.th + 8 * i, f.t);
+  ld_f8(R.m + 8 * i, f.m);
+  ld_f8(R.v + 8 * i, f.v);
 }
 
 template <int MODE, bool CLIP>
 __device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint64_t i,
                                               const AdamScalars& s, float coef) {
   const uint32_t gw[4] = {f.g.x, f.g.y, f.g.z, f.g.w};
-  float tt[8] = {f.t0.x, f.t0.y, f.t0.z, f.t0.w, f.t1.x, f.t1.y, f.t1.z, f.t1.w};
-  float mm[8] = {f.m0.x, f.m0.y, f.m0.z, f.m0.w, f.m1.x, f.m1.y, f.m1.z, f.m1.w};
-  float vv[8] = {f.v0.x, f.v0.y, f.v0.z, f.v0.w, f.v1.x, f.v1.y, f.v1.z, f.v1.w};
   const bool wd = R.wd_on != 0;
 #pragma unroll
   for (int k = 0; k < 8; ++k) {
     const uint32_t w = gw[k >> 1];
     float g = bf16_bits_to_f32((k & 1) ? (w >> 16) : (w & 0xFFFFu));
     if (CLIP) g = __fmul_rn(g, coef);
-    adam_update<MODE>(g, tt[k], mm[k], vv[k], s, wd);
+    adam_update<MODE>(g, f.t[k], f.m[k], f.v[k], s, wd);
   }
-  float4* th = reinterpret_cast<float4*>(R.th) + 2 * i;
-  float4* mp = reinterpret_cast<float4*>(R.m) + 2 * i;
-  float4* vp = reinterpret_cast<float4*>(R.v) + 2 * i;
-  __stcs(th, make_float4(tt[0], tt[1], tt[2], tt[3]));
-  __stcs(th + 1, make_float4(tt[4], tt[5], tt[6], tt[7]));
-  __stcs(mp, make_float4(mm[0], mm[1], mm[2], mm[3]));
-  __stcs(mp + 1, make_float4(mm[4], mm[5], mm[6], mm[7]));
-  __stcs(vp, make_float4(vv[0], vv[1], vv[2], vv[3]));
-  __stcs(vp + 1, make_float4(vv[4], vv[5], vv[6], vv[7]));
+  st_f8(R.th + 8 * i, f.t);
+  st_f8(R.m + 8 * i, f.m);
+  st_f8(R.v + 8 * i, f.v);
   uint4 pk;
-  pk.x = pack_bf16x2_rn(tt[0], tt[1]);
-  pk.y = pack_bf16x2_rn(tt[2], tt[3]);
-  pk.z = pack_bf16x2_rn(tt[4], tt[5]);
-  pk.w = pack_bf16x2_rn(tt[6], tt[7]);
-  __stcs(reinterpret_cast<uint4*>(R.p) + i, pk);
+  pk.x = pack_bf16x2_rn(f.t[0], f.t[1]);
+  pk.y = pack_bf16x2_rn(f.t[2], f.t[3]);
+  pk.z = pack_bf16x2_rn(f.t[4], f.t[5]);
+  pk.w = pack_bf16x2_rn(f.t[6], f.t[7]);
+  st_p8(R.p + 8 * i, pk);
 }
 
 template <int MODE, bool CLIP>
@@ -162,11 +229,12 @@ __device__ __forceinline__ float clip_coef_from(const double* sumsq, double max_
   return static_cast<float>(c);
 }
 
-// K1.  Grid-stride over 8-element vectors of each range, 2 vectors in flight
-// per thread per iteration (all 14 loads issued before any math), then the
-// < 8-element scalar tail.
+// K1.  Grid-stride over 8-element octets of each range, RATEL_K1_UNROLL
+// octets in flight per thread (all their loads issued before any math), then
+// the < 8-element scalar tail.
 template <int MODE, bool CLIP>
-__global__ void __launch_bounds__(kThreads) adam_update_kernel(const __grid_constant__ UpdateParams P) {
+__global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(const __grid_constant__ UpdateParams P) {
+  constexpr int U = RATEL_K1_UNROLL;
   float coef = 1.0f;
   if (CLIP) coef = clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag);
   const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -175,20 +243,191 @@ __global__ void __launch_bounds__(kThreads) adam_update_kernel(const __grid_cons
     const RangeDesc R = P.r[r];
     const uint64_t n8 = R.n >> 3;
     uint64_t i = tid;
-    for (; i + stride < n8; i += 2 * stride) {
-      Frag8 a, b;
-      load8(a, R, i);
-      load8(b, R, i + stride);
-      update_store8<MODE, CLIP>(a, R, i, P.s, coef);
-      update_store8<MODE, CLIP>(b, R, i + stride, P.s, coef);
+    for (; i + (U - 1) * stride < n8; i += U * stride) {
+      Frag8 f[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) load8(f[u], R, i + u * stride);
+#pragma unroll
+      for (int u = 0; u < U; ++u) update_store8<MODE, CLIP>(f[u], R, i + u * stride, P.s, coef);
     }
-    if (i < n8) {
-      Frag8 a;
-      load8(a, R, i);
-      update_store8<MODE, CLIP>(a, R, i, P.s, coef);
+    for (; i < n8; i += stride) {
+      Frag8 f;
+      load8(f, R, i);
+      update_store8<MODE, CLIP>(f, R, i, P.s, coef);
     }
     const uint64_t j = (n8 << 3) + tid;
     if (j < R.n) update_scalar<MODE, CLIP>(R, j, P.s, coef);
+  }
+}
+
+// ---- K1, TMA-staged variant ------------------------------------------------
+// One CTA per SM (persistent).  A producer warp streams each tile's g, theta,
+// m, v into a ring of shared-memory stages with 1-D bulk copies
+// (cp.async.bulk, completion on an mbarrier); consumer warps run the same
+// adam_update() per element from shared memory and write theta, m, v, P16
+// straight to global with 256-bit stores.  Bytes in flight are bounded by the
+// stage ring (RATEL_TMA_STAGES x 14 B x tile), not by registers.
+#ifndef RATEL_TMA_CONSUMER_WARPS
+#define RATEL_TMA_CONSUMER_WARPS 16
+#endif
+#ifndef RATEL_TMA_STAGES
+#define RATEL_TMA_STAGES 3
+#endif
+// How consumers release a stage back to the producer (measured, see
+// profiles/r01_k1_variants.md):  0 lane 0 after __syncwarp -- RACY: the TMA
+// refill can overwrite smem that other lanes' LDS have not read yet (caught
+// by tests with a capped grid); 1 every thread arrives; 2 one arrive per warp
+// AFTER the values were consumed (data dependence makes it safe; fastest);
+// 3 fence.proxy.async then lane 0.
+#ifndef RATEL_TMA_RELEASE
+#define RATEL_TMA_RELEASE 2
+#endif
+constexpr int kTmaConsumerWarps = RATEL_TMA_CONSUMER_WARPS;
+constexpr int kTmaThreads = 32 * (kTmaConsumerWarps + 1);
+constexpr int kTmaTile = kTmaConsumerWarps * 32 * 8;          // elements per tile (1 octet per consumer thread)
+constexpr int kTmaStages = RATEL_TMA_STAGES;
+constexpr uint32_t kTmaStageBytes = kTmaTile * 14;            // g 2 + theta/m/v 12
+constexpr uint32_t kTmaSmemBytes = kTmaStages * kTmaStageBytes + 2 * kTmaStages * 8;
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
+}
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+
+// Tile k of the concatenation of the ranges' vector bodies (n & ~7 each).
+struct TileLoc {
+  int r;
+  uint64_t off;
+  uint32_t len;
+};
+__device__ __forceinline__ TileLoc locate_tile(const UpdateParams& P, uint64_t k) {
+  TileLoc t{0, 0, 0};
+  for (int r = 0; r < P.nr; ++r) {
+    const uint64_t body = P.r[r].n & ~7ull;
+    const uint64_t nt = (body + kTmaTile - 1) / kTmaTile;
+    if (k < nt) {
+      t.r = r;
+      t.off = k * kTmaTile;
+      t.len = static_cast<uint32_t>(body - t.off < (uint64_t)kTmaTile ? body - t.off : kTmaTile);
+      return t;
+    }
+    k -= nt;
+  }
+  t.r = -1;
+  return t;
+}
+
+template <int MODE, bool CLIP>
+__global__ void __launch_bounds__(kTmaThreads, 1) adam_update_tma_kernel(const __grid_constant__ UpdateParams P) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kTmaStages * kTmaStageBytes);
+  uint64_t* empty = full + kTmaStages;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kTmaStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], RATEL_TMA_RELEASE == 1 ? 32 * kTmaConsumerWarps : kTmaConsumerWarps);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  uint64_t total = 0;
+  for (int r = 0; r < P.nr; ++r) total += ((P.r[r].n & ~7ull) + kTmaTile - 1) / kTmaTile;
+
+  if (warp == kTmaConsumerWarps) {  // producer
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (uint64_t k = blockIdx.x; k < total; k += gridDim.x) {
+        const TileLoc t = locate_tile(P, k);
+        const RangeDesc& R = P.r[t.r];
+        mbar_wait(&empty[stage], phase ^ 1);
+        uint8_t* base = smem + stage * kTmaStageBytes;
+        mbar_expect_tx(&full[stage], t.len * 14u);
+        bulk_load(base, R.g + t.off, t.len * 2u, &full[stage]);
+        bulk_load(base + kTmaTile * 2, R.th + t.off, t.len * 4u, &full[stage]);
+        bulk_load(base + kTmaTile * 6, R.m + t.off, t.len * 4u, &full[stage]);
+        bulk_load(base + kTmaTile * 10, R.v + t.off, t.len * 4u, &full[stage]);
+        if (++stage == kTmaStages) {
+          stage = 0;
+          phase ^= 1;
+        }
+      }
+    }
+  } else {  // consumers
+    float coef = 1.0f;
+    if (CLIP) coef = clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag);
+    int stage = 0;
+    uint32_t phase = 0;
+    const uint32_t o = threadIdx.x;  // octet within the tile
+    for (uint64_t k = blockIdx.x; k < total; k += gridDim.x) {
+      const TileLoc t = locate_tile(P, k);
+      const RangeDesc& R = P.r[t.r];
+      mbar_wait(&full[stage], phase);
+      const uint8_t* base = smem + stage * kTmaStageBytes;
+      const bool valid = 8 * o < t.len;
+      Frag8 f;
+      if (valid) {
+        f.g = *reinterpret_cast<const uint4*>(base + 16 * o);
+        const float4* th = reinterpret_cast<const float4*>(base + kTmaTile * 2) + 2 * o;
+        const float4* mm = reinterpret_cast<const float4*>(base + kTmaTile * 6) + 2 * o;
+        const float4* vv = reinterpret_cast<const float4*>(base + kTmaTile * 10) + 2 * o;
+        const float4 t0 = th[0], t1 = th[1], m0 = mm[0], m1 = mm[1], v0 = vv[0], v1 = vv[1];
+        f.t[0] = t0.x; f.t[1] = t0.y; f.t[2] = t0.z; f.t[3] = t0.w;
+        f.t[4] = t1.x; f.t[5] = t1.y; f.t[6] = t1.z; f.t[7] = t1.w;
+        f.m[0] = m0.x; f.m[1] = m0.y; f.m[2] = m0.z; f.m[3] = m0.w;
+        f.m[4] = m1.x; f.m[5] = m1.y; f.m[6] = m1.z; f.m[7] = m1.w;
+        f.v[0] = v0.x; f.v[1] = v0.y; f.v[2] = v0.z; f.v[3] = v0.w;
+        f.v[4] = v1.x; f.v[5] = v1.y; f.v[6] = v1.z; f.v[7] = v1.w;
+      }
+#if RATEL_TMA_RELEASE == 0
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[stage]);  // the stage's data is in registers now
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+#elif RATEL_TMA_RELEASE == 1
+      mbar_arrive(&empty[stage]);                 // every consumer thread arrives
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+#elif RATEL_TMA_RELEASE == 2
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[stage]);  // after the values were consumed
+#else
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[stage]);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+#endif
+      if (++stage == kTmaStages) {
+        stage = 0;
+        phase ^= 1;
+      }
+    }
+    // scalar tails (< 8 elements per range), CTA 0
+    if (blockIdx.x == 0) {
+      for (int r = 0; r < P.nr; ++r) {
+        const uint64_t j = (P.r[r].n & ~7ull) + threadIdx.x;
+        if (j < P.r[r].n) update_scalar<MODE, CLIP>(P.r[r], j, P.s, coef);
+      }
+    }
   }
 }
 

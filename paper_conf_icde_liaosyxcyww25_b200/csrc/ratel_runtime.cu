@@ -153,9 +153,33 @@ const uint16_t* grad_ptr(const ratel_range& r, const Slice& s) {
 }
 
 // ------------------------------------------------------------------ launches
+#ifndef RATEL_K1_TMA
+#define RATEL_K1_TMA 1
+#endif
+
 template <int MODE, bool CLIP>
 void launch_k1(const UpdateParams& P, unsigned grid) {
+#if RATEL_K1_TMA
+  (void)grid;
+  uint64_t tiles = 0;
+  for (int r = 0; r < P.nr; ++r) tiles += ((P.r[r].n & ~7ull) + kTmaTile - 1) / kTmaTile;
+  uint64_t cap = static_cast<uint64_t>(G.sms);
+  if (G.cfg.max_ctas > 0) cap = std::min<uint64_t>(cap, static_cast<uint64_t>(G.cfg.max_ctas));
+  const unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
+  adam_update_tma_kernel<MODE, CLIP><<<g, kTmaThreads, kTmaSmemBytes, G.s_opt>>>(P);
+#else
   adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, G.s_opt>>>(P);
+#endif
+}
+
+template <int MODE, bool CLIP>
+cudaError_t prepare_k1() {
+#if RATEL_K1_TMA
+  return cudaFuncSetAttribute(adam_update_tma_kernel<MODE, CLIP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              static_cast<int>(kTmaSmemBytes));
+#else
+  return cudaSuccess;
+#endif
 }
 
 int launch_update(const RangeDesc* rd, int nr) {
@@ -416,6 +440,10 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   else
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, adam_update_kernel<RATEL_ADAM_L2, false>, kThreads, 0));
   G.k1_grid = G.sms * std::max(occ, 1);
+  CK((prepare_k1<RATEL_ADAMW, false>()));
+  CK((prepare_k1<RATEL_ADAMW, true>()));
+  CK((prepare_k1<RATEL_ADAM_L2, false>()));
+  CK((prepare_k1<RATEL_ADAM_L2, true>()));
   if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
   G.k2_grid = G.sms * 2;
   CK(cudaMalloc(&G.d_sumsq, 2 * sizeof(double)));
@@ -592,6 +620,7 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
   s.eps = static_cast<float>(eps);
   s.decay = static_cast<float>(1.0 - lr * weight_decay);
   s.wd = static_cast<float>(weight_decay);
+  s.wd_d = weight_decay;
   G.armed = true;
   G.last_step = step;
   if (G.cfg.max_grad_norm > 0.0) {

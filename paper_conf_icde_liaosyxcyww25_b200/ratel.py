@@ -68,11 +68,13 @@ class ratel_range(ctypes.Structure):
     ]
 
 
-def _load():
-    if not os.path.exists(_LIB_PATH):
-        raise ImportError(f"{_LIB_PATH} is missing: build it with "
+def load_library(path: str = _LIB_PATH):
+    """Load a libratel.so build and declare its signatures (tools load
+    build-variant copies through this; the package uses the in-tree one)."""
+    if not os.path.exists(path):
+        raise ImportError(f"{path} is missing: build it with "
                           "`python -c 'import __graft_entry__ as g; g.build()'` (no CPU fallback exists)")
-    lib = ctypes.CDLL(_LIB_PATH)
+    lib = ctypes.CDLL(path)
     P, I, U64, D = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint64, ctypes.c_double
     sig = {
         "ratel_default_config": (None, [ctypes.POINTER(ratel_config)]),
@@ -103,7 +105,7 @@ def _load():
     return lib
 
 
-_lib = _load()
+_lib = load_library()
 LIB_PATH = _LIB_PATH
 
 

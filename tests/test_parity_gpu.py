@@ -171,12 +171,21 @@ def test_pinned_host_bitwise_equals_device(cuda_dev, depth, staging, tile):
     assert_bitwise(snapshot(a), snapshot(b))
 
 
-def test_max_ctas_cap_bitwise(cuda_dev):
+@pytest.mark.parametrize("max_ctas", [1, 3, 37])
+def test_max_ctas_cap_bitwise(cuda_dev, max_ctas):
+    """A capped grid makes every CTA cycle its shared-memory stage ring many
+    times (the TMA pipeline's phase/release logic); results must not move."""
     a = _fresh(SIZES, cuda_dev)
     run(a, 2, check_every=False)
     b = _fresh(SIZES, cuda_dev)
-    run(b, 2, check_every=False, max_ctas=3)
+    run(b, 2, check_every=False, max_ctas=max_ctas)
     assert_bitwise(snapshot(a), snapshot(b))
+
+
+def test_large_block_ring_wraps_vs_oracle(cuda_dev):
+    """20M + 5 elements, two ranges: ~33 tiles per CTA at the full grid."""
+    b = GpuBlock(0, [20_000_005, 4_096 * 7 + 3], cuda_dev)
+    run([b], 3)
 
 
 def test_overlapped_with_backward_stream(cuda_dev):
@@ -200,8 +209,6 @@ def test_overlapped_with_backward_stream(cuda_dev):
                         x = (x @ x).clamp_(-1, 1)          # "backward" work
                     for i, hg in enumerate(host[b.id]):
                         b.g16[i][:hg.numel()].copy_(hg, non_blocking=True)
-                    for gt in b.g16:
-                        gt.record_stream(torch.cuda.ExternalStream(R.ratel_optimizer_stream()))
                     R.ratel_offload_grad_chunk(b.id, bwd)
             R.ratel_sync(torch.cuda.current_stream())
             torch.cuda.synchronize()
