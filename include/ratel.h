@@ -157,6 +157,16 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
  * is not registered. */
 int ratel_offload_grad_chunk(int block_id, void* stream);
 
+/* Orders `stream` (cudaStream_t) after the update of block `block_id` that
+ * last consumed its gradient: once it returns, work on `stream` may overwrite
+ * that block's grad buffer (and read its P16 slice).  This is what lets a
+ * caller recycle a small ring of gradient buffers during backward -- the
+ * memory side of active gradient offloading: a block's G16 is dead as soon as
+ * its handler ran.  RATEL_ESTATE if the block was handed off
+ * in the current step but its update is not enqueued yet (deferred mode) or
+ * it is not registered. */
+int ratel_block_wait(int block_id, void* stream);
+
 /* Ends the step: `stream` (cudaStream_t) is ordered after every update,
  * write-back and all-gather of the step, so the next forward on it reads the
  * updated P16 (no staleness, footnote 4 P:L1147-1152).  stream == NULL

@@ -453,33 +453,45 @@ __device__ __forceinline__ double block_sum(double x) {
 }
 
 // K2.  Per-CTA partial of sum(g^2): g^2 is exact in fp32 for a bf16 g, the
-// accumulation is in double.  One slot per CTA, no atomics.
+// accumulation is in double (four independent accumulators, four 16-byte
+// loads in flight per thread).  One slot per CTA, no atomics: the result is
+// a fixed function of the grid, so it is reproducible run to run.
+__device__ __forceinline__ double sumsq8(uint4 w) {
+  const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
+  double d = 0.0;
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    const float lo = bf16_bits_to_f32(ws[k] & 0xFFFFu), hi = bf16_bits_to_f32(ws[k] >> 16);
+    d += static_cast<double>(__fmul_rn(lo, lo));
+    d += static_cast<double>(__fmul_rn(hi, hi));
+  }
+  return d;
+}
+
 __global__ void __launch_bounds__(kThreads) grad_sumsq_kernel(const __grid_constant__ SumsqParams P) {
   const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-  double acc = 0.0;
+  double a0 = 0.0, a1 = 0.0, a2 = 0.0, a3 = 0.0;
   for (int r = 0; r < P.nr; ++r) {
-    const uint16_t* g = P.g[r];
+    const uint4* g = reinterpret_cast<const uint4*>(P.g[r]);
     const uint64_t n = P.n[r], n8 = n >> 3;
-    for (uint64_t i = tid; i < n8; i += stride) {
-      const uint4 w = __ldcs(reinterpret_cast<const uint4*>(g) + i);
-      const uint32_t ws[4] = {w.x, w.y, w.z, w.w};
-      double d = 0.0;
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        const float lo = bf16_bits_to_f32(ws[k] & 0xFFFFu), hi = bf16_bits_to_f32(ws[k] >> 16);
-        d += static_cast<double>(__fmul_rn(lo, lo));
-        d += static_cast<double>(__fmul_rn(hi, hi));
-      }
-      acc += d;
+    uint64_t i = tid;
+    for (; i + 3 * stride < n8; i += 4 * stride) {
+      const uint4 w0 = __ldcs(g + i), w1 = __ldcs(g + i + stride);
+      const uint4 w2 = __ldcs(g + i + 2 * stride), w3 = __ldcs(g + i + 3 * stride);
+      a0 += sumsq8(w0);
+      a1 += sumsq8(w1);
+      a2 += sumsq8(w2);
+      a3 += sumsq8(w3);
     }
+    for (; i < n8; i += stride) a0 += sumsq8(__ldcs(g + i));
     const uint64_t j = (n8 << 3) + tid;
     if (j < n) {
-      const float x = bf16_bits_to_f32(g[j]);
-      acc += static_cast<double>(__fmul_rn(x, x));
+      const float x = bf16_bits_to_f32(P.g[r][j]);
+      a0 += static_cast<double>(__fmul_rn(x, x));
     }
   }
-  const double t = block_sum(acc);
+  const double t = block_sum((a0 + a1) + (a2 + a3));
   if (threadIdx.x == 0) P.partials[blockIdx.x] = t;
 }
 

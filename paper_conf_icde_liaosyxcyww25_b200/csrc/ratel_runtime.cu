@@ -445,7 +445,7 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK((prepare_k1<RATEL_ADAM_L2, false>()));
   CK((prepare_k1<RATEL_ADAM_L2, true>()));
   if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
-  G.k2_grid = G.sms * 2;
+  G.k2_grid = G.sms * 4;
   CK(cudaMalloc(&G.d_sumsq, 2 * sizeof(double)));
   CK(cudaMemset(G.d_sumsq, 0, 2 * sizeof(double)));
   CK(cudaHostAlloc(&G.h_flag, sizeof(int), cudaHostAllocMapped));
@@ -652,6 +652,17 @@ int ratel_offload_grad_chunk(int block_id, void* stream) {
     RK(enqueue_block(B));  // active message: handler runs now, overlapping backward
   else
     G.pending.push_back(block_id);
+  return RATEL_OK;
+}
+
+int ratel_block_wait(int block_id, void* stream) {
+  RK(entry());
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
+    return set_error(RATEL_ESTATE, "ratel_block_wait: block %d is not registered", block_id);
+  const Block& B = G.blocks[block_id];
+  if (B.handed_off && !B.enqueued)
+    return set_error(RATEL_ESTATE, "ratel_block_wait: block %d's update is not enqueued yet", block_id);
+  CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), B.ev_done, 0));
   return RATEL_OK;
 }
 

@@ -84,6 +84,7 @@ def load_library(path: str = _LIB_PATH):
         "ratel_adam_step": (I, [D, D, D, D, D, ctypes.c_int64]),
         "ratel_offload_grad_chunk": (I, [I, P]),
         "ratel_sync": (I, [P]),
+        "ratel_block_wait": (I, [I, P]),
         "ratel_finalize": (I, []),
         "ratel_last_error": (ctypes.c_char_p, []),
         "ratel_padded_numel": (U64, [U64, I]),
@@ -159,6 +160,10 @@ def ratel_adam_step(lr: float, beta1: float, beta2: float, eps: float, weight_de
 
 def ratel_offload_grad_chunk(block_id: int, stream=None) -> None:
     _check(_lib.ratel_offload_grad_chunk(block_id, _stream(stream)))
+
+
+def ratel_block_wait(block_id: int, stream=None) -> None:
+    _check(_lib.ratel_block_wait(block_id, _stream(stream)))
 
 
 def ratel_sync(stream=None) -> None:

@@ -339,3 +339,87 @@ def test_device_generator_matches_synth(cuda_dev):
         assert np.array_equal(g.cpu().numpy().view(np.uint16), synth.grad16(n, step, blk, start=start))
         assert np.array_equal(th.cpu().numpy().view(np.uint32),
                               synth.theta0(n, blk, start=start).view(np.uint32))
+
+
+def test_grad_ring_recycling_with_block_wait(cuda_dev):
+    """5 blocks share a ring of 2 gradient buffers: the backward stream waits
+    (ratel_block_wait) for the update that consumed a slot before writing the
+    next block's gradient into it -- the AGO memory pattern."""
+    sizes = [70_001, 65_536, 40_000, 33_333, 8]
+    blocks = _fresh([[n] for n in sizes], cuda_dev)
+    cap = max(R.ratel_padded_numel(n, 1) for n in sizes)
+    ring = [torch.zeros(cap, dtype=torch.bfloat16, device=cuda_dev) for _ in range(2)]
+    for b in blocks:
+        b.g16 = [ring[b.id % 2]]
+    with ratel_lib():
+        for b in blocks:
+            b.register()
+        bwd = torch.cuda.Stream()
+        for t in (1, 2, 3):
+            grads = {b.id: b.grads_np(t) for b in blocks}
+            host = {b.id: u16_to_torch(grads[b.id][0], "cpu").pin_memory() for b in blocks}
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            with torch.cuda.stream(bwd):
+                order = sorted(blocks, key=lambda b: -b.id)
+                for j, b in enumerate(order):
+                    if j >= 2:
+                        R.ratel_block_wait(b.id + 2, bwd)      # slot's previous block consumed
+                    slot = ring[b.id % 2]
+                    slot[:host[b.id].numel()].copy_(host[b.id], non_blocking=True)
+                    R.ratel_offload_grad_chunk(b.id, bwd)
+            R.ratel_sync(torch.cuda.current_stream())
+            torch.cuda.synchronize()
+            oracle_step(blocks, t, grads)
+            for b in blocks:
+                check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne, what=f"t{t} b{b.id}")
+        # deferred arming: the update is not enqueued yet -> waiting is refused
+        R.ratel_offload_grad_chunk(0, None)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_block_wait(0, None)
+        assert e.value.code == R.RATEL_ESTATE
+        R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, 4)
+        R.ratel_block_wait(0, None)
+        for b in blocks[1:]:
+            R.ratel_offload_grad_chunk(b.id, None)
+        R.ratel_sync(None)
+
+
+def test_fullsize_13b_blocks_sampled_vs_oracle(cuda_dev):
+    """BASELINE configs[1] block size (314,639,360 params, h = 5120) in the
+    bench's launch configuration, inputs from the device generator: sampled
+    elements vs the oracle computed one by one; no-staleness on every element."""
+    h = 5120
+    n = 12 * h * h + 13 * h
+    nblk, steps = 2, 3
+    idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(n - 64, n),
+                                    np.random.default_rng(3).integers(0, n, 200_000)])).astype(np.uint64)
+    state = []
+    with ratel_lib():
+        g = torch.empty(n, dtype=torch.bfloat16, device=cuda_dev)
+        for b in range(nblk):
+            th = torch.empty(n, dtype=torch.float32, device=cuda_dev)
+            R.ratel_gen_theta0(th.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, b))
+            m = torch.zeros(n, device=cuda_dev)
+            v = torch.zeros(n, device=cuda_dev)
+            p = torch.zeros(n, dtype=torch.bfloat16, device=cuda_dev)
+            state.append((p, th, m, v))
+            R.ratel_register_block(b, [R.make_range(p, g, th, m, v, n)], R.RATEL_DEVICE)
+        refs = [oracle.Range.fresh(synth.theta0_at(idx, block=b)) for b in range(nblk)]
+        for t in range(1, steps + 1):
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            for b in reversed(range(nblk)):
+                # the single grad buffer is rewritten per block: wait for the previous consumer
+                if b < nblk - 1:
+                    R.ratel_block_wait(b + 1, None)
+                R.ratel_gen_grad16(g.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, b))
+                R.ratel_offload_grad_chunk(b, None)
+            R.ratel_sync(None)
+            for b in range(nblk):
+                oracle.adam_range(refs[b], synth.grad16_at(idx, step=t, block=b), oracle.hparams(step=t))
+        ii = torch.from_numpy(idx.astype(np.int64)).to(cuda_dev)
+        for b in range(nblk):
+            p, th, m, v = state[b]
+            got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
+                       p16=torch_to_u16(p[ii]))
+            check_range(got, refs[b], own_rne=oracle.bf16_rne, what=f"13B block {b}")
+            assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
