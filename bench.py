@@ -240,6 +240,57 @@ class Model:
         torch.cuda.synchronize()
 
 
+def linears(h):
+    # (out, in) of QKV, proj, fc1, fc2 in the block's flat P16 buffer
+    return [(3 * h, h), (h, h), (4 * h, h), (h, 4 * h)]
+
+
+class SynthBackward:
+    """Synthetic backward for the overlap measurement (harness, cuBLAS via
+    torch): per block the dX and dW GEMMs of its four linears (4*P_blk*T
+    FLOPs), dW written into the block's grad-ring slot."""
+    def __init__(self, dev, h, tokens, p16_views, grad_ring, vocab_rows):
+        import torch
+        self.h, self.T = h, tokens
+        self.dev = dev
+        g = torch.Generator(device=dev)
+        g.manual_seed(1)
+        mk = lambda *s: (torch.randn(*s, device=dev, dtype=torch.bfloat16, generator=g) * 0.01)
+        self.X = {1: mk(tokens, h), 4: mk(tokens, 4 * h)}
+        self.dY = {3: mk(tokens, 3 * h), 1: mk(tokens, h), 4: mk(tokens, 4 * h)}
+        self.dX = torch.empty(tokens, 4 * h, device=dev, dtype=torch.bfloat16)
+        self.p16 = p16_views
+        self.ring = grad_ring
+        self.vocab_rows = vocab_rows
+        self.dYv = mk(2048, vocab_rows) if vocab_rows else None
+
+    def block(self, b, slot):
+        """GEMMs of block b; dW into ring slot `slot` (flat, same layout as P16)."""
+        import torch
+        h, T = self.h, self.T
+        P = self.p16[b]
+        G = self.ring[slot]
+        if b == len(self.p16) - 1 and self.vocab_rows:
+            # embedding block (tied token embedding / LM head): dW[V, h] =
+            # dY^T X accumulated over 2048-token chunks of the logits grad
+            V = self.vocab_rows
+            out = G[:V * h].view(V, h)
+            X = self.X[1]
+            out.zero_()
+            for t0 in range(0, T, 2048):
+                t1 = min(T, t0 + 2048)
+                out.addmm_(self.dYv[:t1 - t0].t(), X[t0:t1])
+            return
+        off = 0
+        for (o, i) in linears(h):
+            W = P[off:off + o * i].view(o, i)
+            X = self.X[i // h]
+            dY = self.dY[o // h]
+            torch.mm(dY, W, out=self.dX[:, :i])                          # dX = dY W
+            torch.mm(dY.t(), X, out=G[off:off + o * i].view(o, i))         # dW = dY^T X
+            off += o * i
+
+
 def init_lib(R, torch, dev_index, rank, world, cfg):
     uid = None
     if world > 1:
@@ -257,6 +308,49 @@ def step_once(R, t, order, stream):
     for b in order:
         R.ratel_offload_grad_chunk(b, stream)
     R.ratel_sync(stream)
+
+
+def overlap_probe(args, R, torch, dev, model, sizes, order, t0):
+    """AGO overlapped with a synthetic backward of `args.overlap_tokens`
+    tokens vs the backward alone (Fig. 7 analog)."""
+    L, h = SHAPES[args.shape]
+    ring = model.grad_ring
+    vocab = VOCAB if len(sizes) == L + 1 else 0
+    bw = SynthBackward(dev, h, args.overlap_tokens, model.p16, ring, vocab)
+    s = torch.cuda.Stream(device=dev, priority=-2)
+    nr = len(ring)
+    t = [t0]
+
+    def bwd_only():
+        with torch.cuda.stream(s):
+            for b in order:
+                bw.block(b, b % nr)
+
+    def ago():
+        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+        t[0] += 1
+        with torch.cuda.stream(s):
+            for j, b in enumerate(order):
+                if j >= nr:
+                    R.ratel_block_wait(b + nr, s)       # ring slot consumed
+                bw.block(b, b % nr)
+                R.ratel_offload_grad_chunk(b, s)
+        R.ratel_sync(s)
+
+    res = {}
+    for name, fn in (("bwd", bwd_only), ("ago", ago)):
+        fn()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        for _ in range(2):
+            fn()
+        e1.record(s)
+        e1.synchronize()
+        res[name] = e0.elapsed_time(e1) / 2
+    del bw
+    torch.cuda.empty_cache()
+    return res, t[0]
 
 
 def timed_steps(R, torch, order, stream, t0, K, pre_step=None, post_step=None):
@@ -376,6 +470,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--oracle-sample", type=int, default=1 << 25)
+    ap.add_argument("--overlap-tokens", type=int, default=8192, help="0 disables the AGO overlap probe")
     args = ap.parse_args()
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -450,6 +545,18 @@ def main():
                 "launches": k1_n, "avg_launch_ms": k1_ms / max(k1_n, 1),
                 "k1_share_of_step": (k1_ms / args.steps) / (ms / args.steps),
                 "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
+        overlap = None
+        if args.overlap_tokens > 0 and world == 1 and args.residency == "device" and args.clip == 0:
+            try:
+                o, t = overlap_probe(args, R, torch, dev, model, sizes, order, t + args.steps)
+                opt_ms = ms / args.steps
+                overlap = {"tokens": args.overlap_tokens, "backward_ms": o["bwd"], "ago_step_ms": o["ago"],
+                           "optimizer_alone_ms": opt_ms, "exposed_optimizer_ms": o["ago"] - o["bwd"],
+                           "hidden_fraction": 1.0 - (o["ago"] - o["bwd"]) / opt_ms,
+                           "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)",
+                           "grad_ring": len(model.grad_ring)}
+            except Exception as ex:
+                overlap = {"error": repr(ex)[:300]}
         del model
         R.ratel_finalize()
         torch.cuda.empty_cache()
@@ -478,7 +585,7 @@ def main():
                     "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
                     "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                     "config": cfgd, "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
-                    "clocks": clocks, "gpu_launches": launches,
+                    "clocks": clocks, "gpu_launches": launches, "overlap": overlap,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
             print(json.dumps(line), flush=True)
     finally:

@@ -1,0 +1,170 @@
+"""PyTorch-facing wrappers named after the paper's user API.
+
+PAPER.md Fig. 4 and §IV-E: the user wraps setup
+in ``with Ratel_init():``, calls ``Ratel_hook(model)``, wraps the optimizer
+with ``Ratel_Optimizer(...)`` and drops ``optimizer.step()`` -- each block's
+update runs when its gradient is complete.  Here:
+
+    with Ratel_init():                                   # ratel_init / finalize
+        opt = Ratel_Optimizer(blocks, lr=1e-3, ...)      # flat buffers + register
+        Ratel_hook(opt)                                  # per-block hand-off hooks
+        for x in data:
+            opt.begin_step()            # arm step t (AGO: before backward)
+            loss = model(x); loss.backward()   # blocks handed off as grads complete
+            opt.end_step()              # hand off stragglers, ratel_sync(stream)
+
+`blocks` is a list of parameter lists, one per transformer block, in forward
+order (backward produces them in reverse).  The wrapper owns one
+flat bf16 P16 buffer, one flat bf16 G16 buffer and fp32 master/m/v per range
+(a block has a weight-decay range and a no-decay range for biases/norms); the
+model's parameters become bf16 views of P16 and their ``.grad`` views of G16,
+so autograd accumulates straight into the buffers the library reads.  The
+hand-off is a post-accumulate-grad hook with a per-block countdown.  All
+arithmetic is in libratel.so; this module only arranges memory and calls.
+One backward per step (no gradient accumulation across micro-batches).
+"""
+from __future__ import annotations
+
+import contextlib
+
+import torch
+
+from . import ratel as R
+
+
+@contextlib.contextmanager
+def Ratel_init(device: int | None = None, **cfg_kw):
+    """Initialise the library for this process (multi-GPU: torch.distributed
+    must be initialised; the NCCL id is broadcast over it)."""
+    from . import dist as rdist
+    dev = torch.cuda.current_device() if device is None else device
+    cfg = R.ratel_default_config()
+    for k, v in cfg_kw.items():
+        setattr(cfg, k, v)
+    rdist.init_distributed(dev, cfg)
+    try:
+        yield cfg
+    finally:
+        torch.cuda.synchronize()
+        R.ratel_finalize()
+
+
+class _Range:
+    def __init__(self, params, apply_wd, world, rank, dev, residency):
+        self.params = params
+        self.numel = sum(p.numel() for p in params)
+        cap = R.ratel_padded_numel(self.numel, world)
+        beg, end = R.ratel_rank_slice(self.numel, world, rank)
+        self.p16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+        self.g16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+        flat32 = torch.cat([p.detach().reshape(-1).to(torch.float32) for p in params]).to(dev)
+        s = max(end - beg, 8)
+        if residency == "device":
+            mk = lambda: torch.zeros(s, dtype=torch.float32, device=dev)
+        else:
+            mk = lambda: torch.zeros(s, dtype=torch.float32).pin_memory()
+        self.master, self.m, self.v = mk(), mk(), mk()
+        if end > beg:
+            self.master[:end - beg].copy_(flat32[beg:end])
+        self.p16[:self.numel].copy_(flat32.to(torch.bfloat16))
+        off = 0
+        for p in params:  # parameters become views of the flat buffers
+            k = p.numel()
+            p.data = self.p16[off:off + k].view(p.shape)
+            p.grad = self.g16[off:off + k].view(p.shape)
+            off += k
+        self.apply_wd = apply_wd
+        self.slice = (beg, end)
+
+    def ratel_range(self):
+        return R.make_range(self.p16, self.g16, self.master, self.m, self.v, self.numel, int(self.apply_wd))
+
+
+class Ratel_Optimizer:
+    """AdamW (or Adam-L2) over flat per-block buffers, driven by hand-offs."""
+
+    def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,
+                 residency="device", no_decay=None, first_block_id=0):
+        import torch.distributed as dist
+        distributed = dist.is_available() and dist.is_initialized()
+        world = dist.get_world_size() if distributed else 1
+        rank = dist.get_rank() if distributed else 0
+        dev = torch.device("cuda", torch.cuda.current_device())
+        no_decay = no_decay or (lambda p: p.ndim <= 1)
+        self.lr, self.betas, self.eps, self.weight_decay = lr, betas, eps, weight_decay
+        self.t = 0
+        self.blocks = []
+        self.block_ids = []
+        for j, params in enumerate(blocks):
+            params = [p for p in params if p.requires_grad]
+            if not params:
+                continue
+            groups = [([p for p in params if not no_decay(p)], True), ([p for p in params if no_decay(p)], False)]
+            ranges = [_Range(ps, wd, world, rank, dev, residency) for ps, wd in groups if ps]
+            bid = first_block_id + j
+            R.ratel_register_block(bid, [r.ratel_range() for r in ranges],
+                                   R.RATEL_DEVICE if residency == "device" else R.RATEL_PINNED_HOST)
+            self.blocks.append(ranges)
+            self.block_ids.append(bid)
+        self._pending = {}
+        self._handed = set()
+        self._hooks = []
+
+    # ------------------------------------------------------------ Ratel_hook
+    def install_hooks(self):
+        for bid, ranges in zip(self.block_ids, self.blocks):
+            params = [p for r in ranges for p in r.params]
+            for p in params:
+                self._hooks.append(p.register_post_accumulate_grad_hook(self._make_hook(bid, len(params))))
+
+    def _make_hook(self, bid, count):
+        def hook(_p):
+            left = self._pending.get(bid, count) - 1
+            self._pending[bid] = left
+            if left == 0 and bid not in self._handed:
+                self._handed.add(bid)
+                # the active message: gradient complete on the stream backward used
+                R.ratel_offload_grad_chunk(bid, torch.cuda.current_stream())
+        return hook
+
+    # ------------------------------------------------------------- a step
+    def begin_step(self, lr=None, weight_decay=None):
+        """Zero the grad buffers and arm step t (before backward = AGO)."""
+        for ranges in self.blocks:
+            for r in ranges:
+                r.g16.zero_()
+                for p in r.params:  # autograd must keep accumulating into our views
+                    assert p.grad is not None and p.grad.data_ptr() >= r.g16.data_ptr()
+        self.t += 1
+        if lr is not None:
+            self.lr = lr
+        if weight_decay is not None:
+            self.weight_decay = weight_decay
+        self._pending.clear()
+        self._handed.clear()
+        R.ratel_adam_step(self.lr, self.betas[0], self.betas[1], self.eps, self.weight_decay, self.t)
+
+    def end_step(self):
+        """Hand off blocks whose hooks did not fire (unused params) and order
+        the current stream after every update (no staleness)."""
+        s = torch.cuda.current_stream()
+        for bid in self.block_ids:
+            if bid not in self._handed:
+                self._handed.add(bid)
+                R.ratel_offload_grad_chunk(bid, s)
+        R.ratel_sync(s)
+
+    def state(self, block_index: int):
+        """(master, exp_avg, exp_avg_sq, p16, g16) flat views of each range of a block."""
+        return [(r.master, r.m, r.v, r.p16, r.g16) for r in self.blocks[block_index]]
+
+    def remove_hooks(self):
+        for h in self._hooks:
+            h.remove()
+        self._hooks.clear()
+
+
+def Ratel_hook(optimizer: Ratel_Optimizer) -> Ratel_Optimizer:
+    """Install the per-block hand-off hooks (Fig. 4's `Ratel_hook(model)`)."""
+    optimizer.install_hooks()
+    return optimizer

@@ -1,0 +1,66 @@
+"""The paper's user API (Fig. 4) on a small bf16 model.
+
+Ratel_init / Ratel_Optimizer / Ratel_hook on three MLP+LayerNorm blocks:
+autograd accumulates into the wrapper's flat G16 buffers, post-accumulate
+hooks hand each block off during backward, and after end_step() every
+range's P32/m/v/P16 must equal the CPU oracle run on the same gradients.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_icde_liaosyxcyww25_b200 as R
+from paper_conf_icde_liaosyxcyww25_b200.api import Ratel_hook, Ratel_init, Ratel_Optimizer
+from tests.tolerance import check_range
+
+pytestmark = pytest.mark.gpu
+
+
+class Block(torch.nn.Module):
+    def __init__(self, d):
+        super().__init__()
+        self.fc1 = torch.nn.Linear(d, 4 * d)
+        self.fc2 = torch.nn.Linear(4 * d, d)
+        self.ln = torch.nn.LayerNorm(d)
+
+    def forward(self, x):
+        return x + self.fc2(torch.nn.functional.gelu(self.fc1(self.ln(x))))
+
+
+def test_paper_api_matches_oracle(cuda_dev):
+    torch.manual_seed(0)
+    d, nb = 96, 3
+    model = torch.nn.Sequential(*[Block(d) for _ in range(nb)]).to(cuda_dev)
+    hp = dict(lr=2e-3, beta1=0.9, beta2=0.99, eps=1e-8, weight_decay=0.05)
+    with Ratel_init():
+        opt = Ratel_Optimizer([list(b.parameters()) for b in model], lr=hp["lr"],
+                              betas=(hp["beta1"], hp["beta2"]), eps=hp["eps"],
+                              weight_decay=hp["weight_decay"])
+        Ratel_hook(opt)
+        assert all(p.dtype == torch.bfloat16 for p in model.parameters())
+        refs = []
+        for bi in range(nb):
+            for (master, m, v, p16, g16), rng in zip(opt.state(bi), opt.blocks[bi]):
+                n = rng.numel
+                refs.append((bi, rng, oracle.Range.fresh(master[:n].cpu().numpy(), int(rng.apply_wd))))
+        x = torch.randn(64, d, device=cuda_dev, dtype=torch.bfloat16)
+        launches0 = R.ratel_launch_count()
+        for t in range(1, 5):
+            opt.begin_step()
+            loss = model(x).float().pow(2).mean()
+            loss.backward()
+            torch.cuda.synchronize()
+            assert len(opt._handed) == nb           # every block handed off by its hooks
+            grads = [r.g16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16) for _, r, _ in refs]
+            opt.end_step()
+            torch.cuda.synchronize()
+            for (bi, rng, ref), g in zip(refs, grads):
+                oracle.adam_range(ref, g, oracle.hparams(step=t, **hp))
+                got = dict(p32=rng.master[:rng.numel].cpu().numpy(), m32=rng.m[:rng.numel].cpu().numpy(),
+                           v32=rng.v[:rng.numel].cpu().numpy(),
+                           p16=rng.p16[:rng.numel].view(torch.int16).cpu().numpy().view(np.uint16))
+                check_range(got, ref, own_rne=oracle.bf16_rne, what=f"api step {t} block {bi}")
+        assert R.ratel_launch_count() - launches0 == 4 * nb
+        opt.remove_hooks()
+        del opt

@@ -36,50 +36,7 @@ import bench  # noqa: E402
 import paper_conf_icde_liaosyxcyww25_b200 as R  # noqa: E402
 
 
-def linears(h):
-    # (out, in) of QKV, proj, fc1, fc2 in the block's flat P16 buffer
-    return [(3 * h, h), (h, h), (4 * h, h), (h, 4 * h)]
-
-
-class SynthBackward:
-    def __init__(self, dev, h, tokens, p16_views, grad_ring, vocab_rows):
-        self.h, self.T = h, tokens
-        self.dev = dev
-        g = torch.Generator(device=dev)
-        g.manual_seed(1)
-        mk = lambda *s: (torch.randn(*s, device=dev, dtype=torch.bfloat16, generator=g) * 0.01)
-        self.X = {1: mk(tokens, h), 4: mk(tokens, 4 * h)}
-        self.dY = {3: mk(tokens, 3 * h), 1: mk(tokens, h), 4: mk(tokens, 4 * h)}
-        self.dX = torch.empty(tokens, 4 * h, device=dev, dtype=torch.bfloat16)
-        self.p16 = p16_views
-        self.ring = grad_ring
-        self.vocab_rows = vocab_rows
-        self.dYv = mk(2048, vocab_rows) if vocab_rows else None
-
-    def block(self, b, slot):
-        """GEMMs of block b; dW into ring slot `slot` (flat, same layout as P16)."""
-        h, T = self.h, self.T
-        P = self.p16[b]
-        G = self.ring[slot]
-        if b == len(self.p16) - 1 and self.vocab_rows:
-            # embedding block (tied token embedding / LM head): dW[V, h] =
-            # dY^T X accumulated over 2048-token chunks of the logits grad
-            V = self.vocab_rows
-            out = G[:V * h].view(V, h)
-            X = self.X[1]
-            out.zero_()
-            for t0 in range(0, T, 2048):
-                t1 = min(T, t0 + 2048)
-                out.addmm_(self.dYv[:t1 - t0].t(), X[t0:t1])
-            return
-        off = 0
-        for (o, i) in linears(h):
-            W = P[off:off + o * i].view(o, i)
-            X = self.X[i // h]
-            dY = self.dY[o // h]
-            torch.mm(dY, W, out=self.dX[:, :i])                          # dX = dY W
-            torch.mm(dY.t(), X, out=G[off:off + o * i].view(o, i))         # dW = dY^T X
-            off += o * i
+from bench import SynthBackward, linears  # noqa: E402,F401
 
 
 def run(args):
