@@ -84,6 +84,13 @@ typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
  * SERIALIZED = Fig. 3a (naive AGO: stage-in, update, write-back in series). */
 typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1 } ratel_staging;
 
+/* Collectives: AUTO = NCCL when world_size > 1; NCCL = also for world_size 1
+ * (a one-rank communicator: exercises the NCCL calls on one GPU); NONE = no
+ * collectives at all -- each rank updates only its slices and the caller
+ * moves the P16 slices itself (simulation/testing of the partition without
+ * NCCL; clipping then uses the rank-local norm). */
+typedef enum { RATEL_COMM_AUTO = 0, RATEL_COMM_NONE = 1, RATEL_COMM_NCCL = 2 } ratel_comm;
+
 typedef struct {
   int mode;               /* ratel_mode; default RATEL_ADAMW */
   double max_grad_norm;   /* > 0 enables the global L2-norm clip (torch clip_grad_norm_); default 0 */
@@ -92,6 +99,7 @@ typedef struct {
   uint64_t tile_elems;    /* pinned-host tile length in elements, multiple of 8; default 1<<24 */
   int max_ctas;           /* cap on the update kernel's grid (0 = SMs x resident CTAs) */
   int timing;             /* 1: bracket every update-kernel launch with CUDA events (ratel_kernel_timing) */
+  int comm;               /* ratel_comm; default RATEL_COMM_AUTO */
 } ratel_config;
 
 /* One contiguous parameter range of a block (a flat tensor, or a block's
@@ -130,7 +138,7 @@ int ratel_get_nccl_unique_id(void* out128);
 /* Creates the optimizer/copy/comm streams (the optimizer stream at the
  * lowest priority), events and, for world_size > 1, the NCCL communicator.
  * device: CUDA ordinal this process drives.  nccl_unique_id: 128 bytes, NULL
- * when world_size == 1.  cfg: NULL = defaults.  RATEL_ESTATE if already
+ * when world_size == 1 (or cfg->comm == RATEL_COMM_NONE).  cfg: NULL = defaults.  RATEL_ESTATE if already
  * initialised; RATEL_ECUDA if no usable device. */
 int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id,
                const ratel_config* cfg);

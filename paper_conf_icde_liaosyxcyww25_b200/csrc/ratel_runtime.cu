@@ -193,7 +193,7 @@ int launch_update(const RangeDesc* rd, int nr) {
   P.nr = nr;
   P.s = G.scal;
   const bool clip = G.cfg.max_grad_norm > 0.0;
-  P.sumsq = G.world > 1 ? G.d_sumsq + 1 : G.d_sumsq;
+  P.sumsq = G.comm != nullptr ? G.d_sumsq + 1 : G.d_sumsq;
   P.max_norm = G.cfg.max_grad_norm;
   P.nonfinite_flag = G.d_flag;
   const uint64_t want = std::max<uint64_t>(1, (max8 + kThreads - 1) / kThreads);
@@ -321,7 +321,7 @@ int enqueue_block(Block& B) {
     }
   }
   CK(cudaEventRecord(B.ev_done, G.s_opt));
-  if (G.world > 1) RK(allgather_block(B));
+  if (G.comm != nullptr) RK(allgather_block(B));
   B.enqueued = true;
   return RATEL_OK;
 }
@@ -333,7 +333,7 @@ int finalize_clip() {
                                                      G.d_sumsq);
   CK(cudaGetLastError());
   ++G.launches;
-  if (G.world > 1)
+  if (G.comm != nullptr)
     NK(g_nccl.AllReduce(G.d_sumsq, G.d_sumsq + 1, 1, ncclFloat64, ncclSum, G.comm, G.s_opt));
   for (int id : G.reg) RK(enqueue_block(G.blocks[id]));
   G.pending.clear();
@@ -369,6 +369,8 @@ int validate_config(const ratel_config& c) {
     return set_error(RATEL_EINVAL, "cfg.staging");
   if (c.tile_elems == 0 || (c.tile_elems & 7u)) return set_error(RATEL_EINVAL, "cfg.tile_elems must be a positive multiple of 8");
   if (c.max_ctas < 0) return set_error(RATEL_EINVAL, "cfg.max_ctas must be >= 0");
+  if (c.comm != RATEL_COMM_AUTO && c.comm != RATEL_COMM_NONE && c.comm != RATEL_COMM_NCCL)
+    return set_error(RATEL_EINVAL, "cfg.comm");
   return RATEL_OK;
 }
 
@@ -452,10 +454,15 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   *G.h_flag = 0;
   CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&G.d_flag), G.h_flag, 0));
   G.blocks.assign(RATEL_MAX_BLOCKS, Block());
-  if (world_size > 1) {
+  const bool want_comm = c.comm == RATEL_COMM_NCCL || (c.comm == RATEL_COMM_AUTO && world_size > 1);
+  if (want_comm) {
     if (const char* m = g_nccl.load()) return set_error(RATEL_ENCCL, "ratel_init: cannot load NCCL: %s", m);
     ncclUniqueId id;
-    memcpy(&id, nccl_unique_id, sizeof id);
+    if (nccl_unique_id != nullptr) {
+      memcpy(&id, nccl_unique_id, sizeof id);
+    } else {  // world_size == 1 with a forced communicator: make our own id
+      NK(g_nccl.GetUniqueId(&id));
+    }
     ncclComm_t comm = nullptr;
     NK(g_nccl.CommInitRank(&comm, world_size, id, rank));
     G.comm = comm;
@@ -476,6 +483,7 @@ void ratel_default_config(ratel_config* cfg) {
   cfg->tile_elems = 1ull << 24;
   cfg->max_ctas = 0;
   cfg->timing = 0;
+  cfg->comm = RATEL_COMM_AUTO;
 }
 
 uint64_t ratel_padded_numel(uint64_t numel, int world_size) {
@@ -508,7 +516,7 @@ int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id,
   if (G.inited) return set_error(RATEL_ESTATE, "ratel_init: already initialised");
   if (world_size < 1 || rank < 0 || rank >= world_size)
     return set_error(RATEL_EINVAL, "ratel_init: need 0 <= rank < world_size");
-  if (world_size > 1 && nccl_unique_id == nullptr)
+  if (world_size > 1 && nccl_unique_id == nullptr && (cfg == nullptr || cfg->comm != RATEL_COMM_NONE))
     return set_error(RATEL_EINVAL, "ratel_init: world_size > 1 needs an NCCL unique id");
   ratel_config c;
   ratel_default_config(&c);
@@ -718,7 +726,7 @@ int ratel_get_grad_sumsq(double* out) {
   if (out == nullptr) return set_error(RATEL_EINVAL, "ratel_get_grad_sumsq: NULL");
   if (!(G.cfg.max_grad_norm > 0.0)) return set_error(RATEL_ESTATE, "ratel_get_grad_sumsq: clipping is off");
   CK(cudaStreamSynchronize(G.s_opt));
-  CK(cudaMemcpy(out, G.world > 1 ? G.d_sumsq + 1 : G.d_sumsq, sizeof(double), cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(out, G.comm != nullptr ? G.d_sumsq + 1 : G.d_sumsq, sizeof(double), cudaMemcpyDeviceToHost));
   return RATEL_OK;
 }
 

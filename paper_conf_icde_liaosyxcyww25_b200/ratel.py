@@ -30,6 +30,9 @@ RATEL_ADAMW = 0
 RATEL_ADAM_L2 = 1
 RATEL_STAGING_PIPELINED = 0
 RATEL_STAGING_SERIALIZED = 1
+RATEL_COMM_AUTO = 0
+RATEL_COMM_NONE = 1
+RATEL_COMM_NCCL = 2
 RATEL_MAX_BLOCKS = 4096
 RATEL_MAX_RANGES_PER_BLOCK = 32
 
@@ -52,6 +55,7 @@ class ratel_config(ctypes.Structure):
         ("tile_elems", ctypes.c_uint64),
         ("max_ctas", ctypes.c_int),
         ("timing", ctypes.c_int),
+        ("comm", ctypes.c_int),
     ]
 
 
