@@ -303,10 +303,16 @@ def init_lib(R, torch, dev_index, rank, world, cfg):
     R.ratel_init(dev_index, rank, world, uid, cfg)
 
 
+ARM_AFTER = False   # --arm after: the deferred "Ratel+ZeRO" order
+
+
 def step_once(R, t, order, stream):
-    R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
+    if not ARM_AFTER:
+        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
     for b in order:
         R.ratel_offload_grad_chunk(b, stream)
+    if ARM_AFTER:
+        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
     R.ratel_sync(stream)
 
 
@@ -385,6 +391,41 @@ def barrier(torch, world):
 
 
 # ------------------------------------------------------------------- e2e
+def host_link_probe(torch, dev, nbytes=1 << 30, reps=3):
+    """Measured duplex host-link bandwidth on this box (pinned H2D and D2H
+    concurrently on two streams): the e2e roofline denominator."""
+    n = nbytes // 4
+    h1 = torch.empty(n, dtype=torch.float32, pin_memory=True)
+    h2 = torch.empty(n, dtype=torch.float32, pin_memory=True)
+    d1 = torch.empty(n, dtype=torch.float32, device=dev)
+    d2 = torch.empty(n, dtype=torch.float32, device=dev)
+    s1, s2 = torch.cuda.Stream(device=dev), torch.cuda.Stream(device=dev)
+    best = {}
+    for name in ("h2d", "d2h", "duplex"):
+        ts = []
+        for _ in range(reps):
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            s1.wait_stream(torch.cuda.current_stream())
+            s2.wait_stream(torch.cuda.current_stream())
+            if name in ("h2d", "duplex"):
+                with torch.cuda.stream(s1):
+                    d1.copy_(h1, non_blocking=True)
+            if name in ("d2h", "duplex"):
+                with torch.cuda.stream(s2):
+                    h2.copy_(d2, non_blocking=True)
+            torch.cuda.current_stream().wait_stream(s1)
+            torch.cuda.current_stream().wait_stream(s2)
+            e1.record()
+            e1.synchronize()
+            ts.append(e0.elapsed_time(e1))
+        moved = nbytes * (2 if name == "duplex" else 1)
+        best[name] = moved / (min(ts) / 1e3) / 1e9
+    del h1, h2, d1, d2
+    return best
+
+
 def run_e2e(args, R, torch, dev, dev_index, rank, world):
     """Pinned-host residency through the C ABI: theta/m/v stream H2D/D2H via
     the library's tile ring; grads H2D from pinned host before each block's
@@ -442,9 +483,12 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
         h2d = (12 * own + 2 * own) * world            # states in + grads in (all ranks)
         d2h = (12 * own) * world + 2 * sum(R.ratel_padded_numel(n, world) for n in sizes) * world
         val = P * K / (ms / 1e3)
+        link = host_link_probe(torch, dev)
+        achieved = (h2d + d2h) / world / (ms / K / 1e3) / 1e9
         res = {"value": val, "unit": UNIT, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                "ms_per_step": ms / K, "steps": K, "params": P, "blocks": n_blk,
-               "host_link_gbs": (h2d + d2h) / world / (ms / K / 1e3) / 1e9,
+               "host_link_gbs": achieved, "host_link_peak_gbs": link["duplex"],
+               "host_link_frac": achieved / link["duplex"], "host_link_probe": link,
                "path": "pinned-host states (tile ring depth %d, %d-elem tiles)" % (cfg.pipeline_depth,
                                                                                    cfg.tile_elems)}
         del model
@@ -471,7 +515,13 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--oracle-sample", type=int, default=1 << 25)
     ap.add_argument("--overlap-tokens", type=int, default=8192, help="0 disables the AGO overlap probe")
+    ap.add_argument("--arm", default="before", choices=["before", "after"],
+                    help="arm before the hand-offs (AGO) or after the last one (deferred)")
+    ap.add_argument("--tile-elems", type=int, default=0)
+    ap.add_argument("--depth", type=int, default=0)
     args = ap.parse_args()
+    global ARM_AFTER
+    ARM_AFTER = args.arm == "after"
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -505,6 +555,10 @@ def main():
     cfg.timing = 1
     cfg.max_ctas = args.max_ctas
     cfg.max_grad_norm = args.clip
+    if args.tile_elems:
+        cfg.tile_elems = args.tile_elems
+    if args.depth:
+        cfg.pipeline_depth = args.depth
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
     try:

@@ -279,6 +279,12 @@ __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(co
 // by tests with a capped grid); 1 every thread arrives; 2 one arrive per warp
 // AFTER the values were consumed (data dependence makes it safe; fastest);
 // 3 fence.proxy.async then lane 0.
+#ifndef RATEL_TMA_EVICT_FIRST
+#define RATEL_TMA_EVICT_FIRST 0
+#endif
+#ifndef RATEL_TMA_CTAS_PER_SM
+#define RATEL_TMA_CTAS_PER_SM 1
+#endif
 #ifndef RATEL_TMA_RELEASE
 #define RATEL_TMA_RELEASE 2
 #endif
@@ -308,8 +314,20 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       " @!p bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
 }
 __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+#if RATEL_TMA_EVICT_FIRST
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+#else
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+#endif
+}
+
+__device__ __forceinline__ void bulk_store(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
+               ::"l"(dst), "r"(smem_u32(src)), "r"(bytes) : "memory");
 }
 
 // Tile k of the concatenation of the ranges' vector bodies (n & ~7 each).
@@ -336,7 +354,7 @@ __device__ __forceinline__ TileLoc locate_tile(const UpdateParams& P, uint64_t k
 }
 
 template <int MODE, bool CLIP>
-__global__ void __launch_bounds__(kTmaThreads, 1) adam_update_tma_kernel(const __grid_constant__ UpdateParams P) {
+__global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_update_tma_kernel(const __grid_constant__ UpdateParams P) {
   extern __shared__ __align__(128) uint8_t smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kTmaStages * kTmaStageBytes);
   uint64_t* empty = full + kTmaStages;
@@ -344,7 +362,8 @@ __global__ void __launch_bounds__(kTmaThreads, 1) adam_update_tma_kernel(const _
   if (threadIdx.x == 0) {
     for (int s = 0; s < kTmaStages; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&empty[s], RATEL_TMA_RELEASE == 1 ? 32 * kTmaConsumerWarps : kTmaConsumerWarps);
+      mbar_init(&empty[s], RATEL_TMA_RELEASE == 1 ? 32 * kTmaConsumerWarps
+                           : (RATEL_TMA_RELEASE == 4 ? 1 : kTmaConsumerWarps));
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -378,6 +397,8 @@ __global__ void __launch_bounds__(kTmaThreads, 1) adam_update_tma_kernel(const _
     if (CLIP) coef = clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag);
     int stage = 0;
     uint32_t phase = 0;
+    int prev_stage = -1;
+    (void)prev_stage;
     const uint32_t o = threadIdx.x;  // octet within the tile
     for (uint64_t k = blockIdx.x; k < total; k += gridDim.x) {
       const TileLoc t = locate_tile(P, k);
@@ -410,17 +431,61 @@ __global__ void __launch_bounds__(kTmaThreads, 1) adam_update_tma_kernel(const _
       if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // after the values were consumed
-#else
+#elif RATEL_TMA_RELEASE == 3
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);
       if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+#else  // 4: results written back into the stage, bulk-stored by one thread
+      if (valid) {
+        const bool wd = R.wd_on != 0;
+        const uint32_t gw[4] = {f.g.x, f.g.y, f.g.z, f.g.w};
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk) {
+          const uint32_t w = gw[kk >> 1];
+          float g = bf16_bits_to_f32((kk & 1) ? (w >> 16) : (w & 0xFFFFu));
+          if (CLIP) g = __fmul_rn(g, coef);
+          adam_update<MODE>(g, f.t[kk], f.m[kk], f.v[kk], P.s, wd);
+        }
+        uint8_t* wb = smem + stage * kTmaStageBytes;
+        float4* th = reinterpret_cast<float4*>(wb + kTmaTile * 2) + 2 * o;
+        float4* mm = reinterpret_cast<float4*>(wb + kTmaTile * 6) + 2 * o;
+        float4* vv = reinterpret_cast<float4*>(wb + kTmaTile * 10) + 2 * o;
+        th[0] = make_float4(f.t[0], f.t[1], f.t[2], f.t[3]);
+        th[1] = make_float4(f.t[4], f.t[5], f.t[6], f.t[7]);
+        mm[0] = make_float4(f.m[0], f.m[1], f.m[2], f.m[3]);
+        mm[1] = make_float4(f.m[4], f.m[5], f.m[6], f.m[7]);
+        vv[0] = make_float4(f.v[0], f.v[1], f.v[2], f.v[3]);
+        vv[1] = make_float4(f.v[4], f.v[5], f.v[6], f.v[7]);
+        uint4 pk;
+        pk.x = pack_bf16x2_rn(f.t[0], f.t[1]);
+        pk.y = pack_bf16x2_rn(f.t[2], f.t[3]);
+        pk.z = pack_bf16x2_rn(f.t[4], f.t[5]);
+        pk.w = pack_bf16x2_rn(f.t[6], f.t[7]);
+        *reinterpret_cast<uint4*>(wb + 16 * o) = pk;
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic smem writes -> async proxy
+      asm volatile("bar.sync 1, %0;" ::"r"(kTmaConsumerWarps * 32) : "memory");
+      if (threadIdx.x == 0) {
+        uint8_t* wb = smem + stage * kTmaStageBytes;
+        bulk_store(R.th + t.off, wb + kTmaTile * 2, t.len * 4u);
+        bulk_store(R.m + t.off, wb + kTmaTile * 6, t.len * 4u);
+        bulk_store(R.v + t.off, wb + kTmaTile * 10, t.len * 4u);
+        bulk_store(R.p + t.off, wb, t.len * 2u);
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");  // previous tile's stores read smem
+        if (prev_stage >= 0) mbar_arrive(&empty[prev_stage]);
+        prev_stage = stage;
+      }
 #endif
       if (++stage == kTmaStages) {
         stage = 0;
         phase ^= 1;
       }
     }
+#if RATEL_TMA_RELEASE == 4
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+#endif
     // scalar tails (< 8 elements per range), CTA 0
     if (blockIdx.x == 0) {
       for (int r = 0; r < P.nr; ++r) {

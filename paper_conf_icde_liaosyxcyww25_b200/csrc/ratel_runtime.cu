@@ -163,7 +163,7 @@ void launch_k1(const UpdateParams& P, unsigned grid) {
   (void)grid;
   uint64_t tiles = 0;
   for (int r = 0; r < P.nr; ++r) tiles += ((P.r[r].n & ~7ull) + kTmaTile - 1) / kTmaTile;
-  uint64_t cap = static_cast<uint64_t>(G.sms);
+  uint64_t cap = static_cast<uint64_t>(G.sms) * RATEL_TMA_CTAS_PER_SM;
   if (G.cfg.max_ctas > 0) cap = std::min<uint64_t>(cap, static_cast<uint64_t>(G.cfg.max_ctas));
   const unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
   adam_update_tma_kernel<MODE, CLIP><<<g, kTmaThreads, kTmaSmemBytes, G.s_opt>>>(P);
