@@ -121,9 +121,10 @@ class ClockSampler:
         if not rows:
             return None
         sm = sorted(float(r[0]) for r in rows if r[0].replace(".", "").isdigit())
+        pw = sorted(float(r[2]) for r in rows if r[2].replace(".", "").isdigit())
         reasons = sorted({self.NAMES[i] for r in rows for i in range(4) if r[3 + i].lower() == "active"})
         return {"sm_mhz": sm[len(sm) // 2] if sm else None, "sm_max_mhz": float(rows[0][1]),
-                "reasons": reasons, "samples": len(rows)}
+                "power_w": pw[len(pw) // 2] if pw else None, "reasons": reasons, "samples": len(rows)}
 
 
 def gpu_uuid(torch, dev):
@@ -453,16 +454,22 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
         s = torch.cuda.Stream(device=dev)
         order = list(reversed(range(n_blk)))
 
+        s_out = torch.cuda.Stream(device=dev)
+
         def one_safe(t):
             R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
             with torch.cuda.stream(s):
                 for b in order:
-                    g_dev[b].copy_(g_host, non_blocking=True)          # G16 host -> device
+                    beg, end = model.slices[b]                         # G16 host -> device
+                    g_dev[b][beg:end].copy_(g_host[beg:end], non_blocking=True)
                     R.ratel_offload_grad_chunk(b, s)
+            with torch.cuda.stream(s_out):
+                for b in order:                                        # P16 device -> host, per block
+                    R.ratel_block_wait(b, s_out)                       # as soon as its update ran
+                    beg, end = model.slices[b]
+                    p_host[b][beg:end].copy_(model.p16[b][beg:end], non_blocking=True)
+            s.wait_stream(s_out)
             R.ratel_sync(s)
-            with torch.cuda.stream(s):
-                for b in range(n_blk):
-                    p_host[b].copy_(model.p16[b], non_blocking=True)  # P16 device -> host
         t = 1
         for _ in range(max(1, min(args.warmup, 2))):
             one_safe(t)
@@ -481,7 +488,7 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
         P = sum(sizes)
         own = sum(e - b for (b, e) in model.slices)
         h2d = (12 * own + 2 * own) * world            # states in + grads in (all ranks)
-        d2h = (12 * own) * world + 2 * sum(R.ratel_padded_numel(n, world) for n in sizes) * world
+        d2h = (12 * own + 2 * own) * world            # states out + this rank's P16 slice (all ranks)
         val = P * K / (ms / 1e3)
         link = host_link_probe(torch, dev)
         achieved = (h2d + d2h) / world / (ms / K / 1e3) / 1e9

@@ -271,14 +271,20 @@ __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(co
 #define RATEL_TMA_CONSUMER_WARPS 16
 #endif
 #ifndef RATEL_TMA_STAGES
-#define RATEL_TMA_STAGES 3
+#define RATEL_TMA_STAGES 4
 #endif
-// How consumers release a stage back to the producer (measured, see
-// profiles/r01_k1_variants.md):  0 lane 0 after __syncwarp -- RACY: the TMA
-// refill can overwrite smem that other lanes' LDS have not read yet (caught
-// by tests with a capped grid); 1 every thread arrives; 2 one arrive per warp
-// AFTER the values were consumed (data dependence makes it safe; fastest);
-// 3 fence.proxy.async then lane 0.
+// How a stage goes back to the producer (measured: profiles/sweeps/,
+// profiles/r01_racecheck_*.log):
+//   0 lane 0 arrives right after __syncwarp -- RACY: the TMA refill overwrote
+//     smem that other lanes' loads had not returned yet (capped-grid tests);
+//   1 every consumer thread arrives (racecheck-clean);
+//   2 lane 0 arrives after the warp CONSUMED the values (correct by data
+//     dependence, but racecheck cannot see that and flags it);
+//   3 fence.proxy.async + lane 0 (flagged by racecheck as well);
+//   4 default: results are written back into the stage and bulk-stored by one
+//     thread (cp.async.bulk global<-shared); that thread releases a stage once
+//     cp.async.bulk.wait_group.read says the store finished reading it.
+//     Racecheck-clean and the fastest (fewer STG instructions).
 #ifndef RATEL_TMA_EVICT_FIRST
 #define RATEL_TMA_EVICT_FIRST 0
 #endif
@@ -286,7 +292,7 @@ __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(co
 #define RATEL_TMA_CTAS_PER_SM 1
 #endif
 #ifndef RATEL_TMA_RELEASE
-#define RATEL_TMA_RELEASE 2
+#define RATEL_TMA_RELEASE 4
 #endif
 constexpr int kTmaConsumerWarps = RATEL_TMA_CONSUMER_WARPS;
 constexpr int kTmaThreads = 32 * (kTmaConsumerWarps + 1);

@@ -110,8 +110,10 @@ def load_library(path: str = _LIB_PATH):
     return lib
 
 
-_lib = load_library()
-LIB_PATH = _LIB_PATH
+# RATEL_LIB lets tools load a build variant (tools/k1_sweep.py builds them);
+# it must name an existing libratel build -- there is no fallback either way.
+LIB_PATH = os.environ.get("RATEL_LIB", _LIB_PATH)
+_lib = load_library(LIB_PATH)
 
 
 def lib():

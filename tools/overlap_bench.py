@@ -22,6 +22,7 @@ import argparse
 import json
 import os
 import sys
+import time
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
@@ -104,18 +105,26 @@ def run(args):
                     one(sch, bw)
                 torch.cuda.synchronize()
                 R.ratel_kernel_timing(reset=True)
+                sampler = bench.ClockSampler(bench.gpu_uuid(torch, dev))
+                time.sleep(0.6)
+                w0 = time.time()
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
                 e0.record(hi)
                 for _ in range(args.steps):
                     one(sch, bw)
                 e1.record(hi)
                 e1.synchronize()
+                sampler.mark(w0, time.time())
+                clk = sampler.stop() or {}
                 k1_ms, _ = R.ratel_kernel_timing(reset=True)
-                times[sch] = (e0.elapsed_time(e1) / args.steps, k1_ms / args.steps)
+                times[sch] = (e0.elapsed_time(e1) / args.steps, k1_ms / args.steps, clk.get("sm_mhz"),
+                              clk.get("power_w"))
                 R.ratel_finalize()
             tb = times["bwd"][0]
             row = {"residency": args.residency, "tokens": tokens, "max_ctas": mc, "blocks": len(sizes),
                    "params": sum(sizes), "bwd_ms": tb, "bwd_tflops": 4 * sum(sizes) * tokens / (tb / 1e3) / 1e12}
+            for sch, v in times.items():
+                row[f"{sch}_sm_mhz"], row[f"{sch}_power_w"] = v[2], v[3]
             if "opt" in times:
                 row["opt_ms"] = times["opt"][0]
                 if args.residency == "host":

@@ -1,0 +1,35 @@
+"""Small AGO steps through the C ABI for compute-sanitizer (memcheck,
+racecheck, synccheck): C1-sized ragged blocks, a capped grid so every CTA
+cycles the TMA stage ring, clip mode, and a pinned-host block."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import torch  # noqa: E402
+
+import paper_conf_icde_liaosyxcyww25_b200 as R  # noqa: E402
+from tests.harness import GpuBlock, ratel_lib  # noqa: E402
+
+
+def run(max_ctas, clip, pinned):
+    dev = torch.device("cuda:0")
+    blocks = [GpuBlock(0, [789_760 + 3], dev, pinned=pinned), GpuBlock(1, [40_001, 17], dev)]
+    with ratel_lib(max_ctas=max_ctas, max_grad_norm=clip, tile_elems=65_536):
+        for b in blocks:
+            b.register()
+        for t in (1, 2):
+            for b in blocks:
+                b.load_grads(t)
+            torch.cuda.synchronize()
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            for b in reversed(blocks):
+                R.ratel_offload_grad_chunk(b.id, None)
+            R.ratel_sync(None)
+
+
+if __name__ == "__main__":
+    run(4, 0.0, False)
+    run(0, 1.0, False)
+    run(2, 0.0, True)
+    print("sanitize_run: done")
