@@ -76,22 +76,29 @@ struct SumsqParams {
 // The per-element update.  Explicit-rounding intrinsics fix the operation
 // sequence (no contraction freedom):
 //   AdamW:   theta = theta*decay            (wd_on)
-//   Adam-L2: g     = fp32(fma(wd, theta, g) in fp64)   (wd_on)
+//   Adam-L2: g     = fp32(g*coef + wd*theta, formed in fp64)   (wd_on)
 // The L2 term is formed in double: g and wd*theta cancel when the gradient
 // balances the decay, and fp32(wd) alone (rel. error 2e-8) would then move
 // g' by more than its own ulp and the update by >1e-5 of its scale near
-// |g'| ~ eps (measured on B200; R3).  One DFMA per element is far
-// inside the ALU budget of this HBM-bound kernel.
+// |g'| ~ eps (measured on B200; R3); with clipping the fp32
+// rounding of g*coef did the same to v (measured).  Two fp64 ops per element
+// are far inside the ALU budget of this HBM-bound kernel.
 //   m     = fma(b1, m, (1-b1)*g)
 //   v     = fma(b2, v, (1-b2)*(g*g))        g*g is exact for a bf16 g
 //   denom = fma(sqrt(v), 1/sqrt(bc2), eps)  == sqrt(v/bc2) + eps
 //   theta = fma(-lr/bc1, m/denom, theta)
-template <int MODE>
-__device__ __forceinline__ void adam_update(float g, float& th, float& m, float& v,
-                                            const AdamScalars& s, bool wd_on) {
+template <int MODE, bool CLIP>
+__device__ __forceinline__ void adam_update(float g, float& th, float& m, float& v, const AdamScalars& s,
+                                            bool wd_on, float coef_f, double coef_d) {
   if (MODE == RATEL_ADAM_L2) {
-    if (wd_on) g = __double2float_rn(__fma_rn(s.wd_d, static_cast<double>(th), static_cast<double>(g)));
+    // g' = g*coef + wd*theta in double, rounded once: the two terms cancel
+    // when the gradient balances the decay (see the comment above).
+    double gd = static_cast<double>(g);
+    if (CLIP) gd *= coef_d;
+    if (wd_on) gd = __fma_rn(s.wd_d, static_cast<double>(th), gd);
+    g = __double2float_rn(gd);
   } else {
+    if (CLIP) g = __fmul_rn(g, coef_f);
     if (wd_on) th = __fmul_rn(th, s.decay);
   }
   m = __fmaf_rn(s.beta1, m, __fmul_rn(s.one_minus_beta1, g));
@@ -187,15 +194,14 @@ __device__ __forceinline__ void load8(Frag8& f, const RangeDesc& R, uint64_t i) 
 
 template <int MODE, bool CLIP>
 __device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint64_t i,
-                                              const AdamScalars& s, float coef) {
+                                              const AdamScalars& s, float coef_f, double coef_d) {
   const uint32_t gw[4] = {f.g.x, f.g.y, f.g.z, f.g.w};
   const bool wd = R.wd_on != 0;
 #pragma unroll
   for (int k = 0; k < 8; ++k) {
     const uint32_t w = gw[k >> 1];
     float g = bf16_bits_to_f32((k & 1) ? (w >> 16) : (w & 0xFFFFu));
-    if (CLIP) g = __fmul_rn(g, coef);
-    adam_update<MODE>(g, f.t[k], f.m[k], f.v[k], s, wd);
+    adam_update<MODE, CLIP>(g, f.t[k], f.m[k], f.v[k], s, wd, coef_f, coef_d);
   }
   st_f8(R.th + 8 * i, f.t);
   st_f8(R.m + 8 * i, f.m);
@@ -210,23 +216,22 @@ __device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint
 
 template <int MODE, bool CLIP>
 __device__ __forceinline__ void update_scalar(const RangeDesc& R, uint64_t j, const AdamScalars& s,
-                                              float coef) {
+                                              float coef_f, double coef_d) {
   float g = bf16_bits_to_f32(R.g[j]);
-  if (CLIP) g = __fmul_rn(g, coef);
   float th = R.th[j], m = R.m[j], v = R.v[j];
-  adam_update<MODE>(g, th, m, v, s, R.wd_on != 0);
+  adam_update<MODE, CLIP>(g, th, m, v, s, R.wd_on != 0, coef_f, coef_d);
   R.th[j] = th;
   R.m[j] = m;
   R.v[j] = v;
   R.p[j] = static_cast<uint16_t>(pack_bf16x2_rn(th, 0.0f) & 0xFFFFu);
 }
 
-__device__ __forceinline__ float clip_coef_from(const double* sumsq, double max_norm, int* flag) {
+__device__ __forceinline__ double clip_coef_from(const double* sumsq, double max_norm, int* flag) {
   const double S = *sumsq;
   double c = max_norm / (sqrt(S) + 1e-6);
   c = (c < 1.0 || isnan(c)) ? c : 1.0;  // torch: clamp(max=1), NaN propagates
   if (flag != nullptr && blockIdx.x == 0 && threadIdx.x == 0) *flag = isfinite(S) ? 0 : 1;
-  return static_cast<float>(c);
+  return c;
 }
 
 // K1.  Grid-stride over 8-element octets of each range, RATEL_K1_UNROLL
@@ -235,8 +240,8 @@ __device__ __forceinline__ float clip_coef_from(const double* sumsq, double max_
 template <int MODE, bool CLIP>
 __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(const __grid_constant__ UpdateParams P) {
   constexpr int U = RATEL_K1_UNROLL;
-  float coef = 1.0f;
-  if (CLIP) coef = clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag);
+  const double coef_d = CLIP ? clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag) : 1.0;
+  const float coef_f = static_cast<float>(coef_d);
   const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
   const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
   for (int r = 0; r < P.nr; ++r) {
@@ -248,15 +253,15 @@ __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(co
 #pragma unroll
       for (int u = 0; u < U; ++u) load8(f[u], R, i + u * stride);
 #pragma unroll
-      for (int u = 0; u < U; ++u) update_store8<MODE, CLIP>(f[u], R, i + u * stride, P.s, coef);
+      for (int u = 0; u < U; ++u) update_store8<MODE, CLIP>(f[u], R, i + u * stride, P.s, coef_f, coef_d);
     }
     for (; i < n8; i += stride) {
       Frag8 f;
       load8(f, R, i);
-      update_store8<MODE, CLIP>(f, R, i, P.s, coef);
+      update_store8<MODE, CLIP>(f, R, i, P.s, coef_f, coef_d);
     }
     const uint64_t j = (n8 << 3) + tid;
-    if (j < R.n) update_scalar<MODE, CLIP>(R, j, P.s, coef);
+    if (j < R.n) update_scalar<MODE, CLIP>(R, j, P.s, coef_f, coef_d);
   }
 }
 
@@ -399,8 +404,8 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
       }
     }
   } else {  // consumers
-    float coef = 1.0f;
-    if (CLIP) coef = clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag);
+    const double coef_d = CLIP ? clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag) : 1.0;
+    const float coef_f = static_cast<float>(coef_d);
     int stage = 0;
     uint32_t phase = 0;
     int prev_stage = -1;
@@ -429,19 +434,19 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
 #if RATEL_TMA_RELEASE == 0
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // the stage's data is in registers now
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
 #elif RATEL_TMA_RELEASE == 1
       mbar_arrive(&empty[stage]);                 // every consumer thread arrives
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
 #elif RATEL_TMA_RELEASE == 2
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // after the values were consumed
 #elif RATEL_TMA_RELEASE == 3
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
 #else  // 4: results written back into the stage, bulk-stored by one thread
       if (valid) {
         const bool wd = R.wd_on != 0;
@@ -450,8 +455,7 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
         for (int kk = 0; kk < 8; ++kk) {
           const uint32_t w = gw[kk >> 1];
           float g = bf16_bits_to_f32((kk & 1) ? (w >> 16) : (w & 0xFFFFu));
-          if (CLIP) g = __fmul_rn(g, coef);
-          adam_update<MODE>(g, f.t[kk], f.m[kk], f.v[kk], P.s, wd);
+          adam_update<MODE, CLIP>(g, f.t[kk], f.m[kk], f.v[kk], P.s, wd, coef_f, coef_d);
         }
         uint8_t* wb = smem + stage * kTmaStageBytes;
         float4* th = reinterpret_cast<float4*>(wb + kTmaTile * 2) + 2 * o;
@@ -496,7 +500,7 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
     if (blockIdx.x == 0) {
       for (int r = 0; r < P.nr; ++r) {
         const uint64_t j = (P.r[r].n & ~7ull) + threadIdx.x;
-        if (j < P.r[r].n) update_scalar<MODE, CLIP>(P.r[r], j, P.s, coef);
+        if (j < P.r[r].n) update_scalar<MODE, CLIP>(P.r[r], j, P.s, coef_f, coef_d);
       }
     }
   }

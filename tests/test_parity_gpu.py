@@ -423,3 +423,28 @@ def test_fullsize_13b_blocks_sampled_vs_oracle(cuda_dev):
                        p16=torch_to_u16(p[ii]))
             check_range(got, refs[b], own_rne=oracle.bf16_rne, what=f"13B block {b}")
             assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
+
+
+def test_max_ranges_and_block_ids(cuda_dev):
+    """A block with RATEL_MAX_RANGES_PER_BLOCK ranges (sizes 1..., mixed wd
+    flags) under the largest block id, next to a one-range block; and the
+    33rd range is rejected."""
+    n_r = R.RATEL_MAX_RANGES_PER_BLOCK
+    sizes = [1 + 37 * i for i in range(n_r)]
+    big = GpuBlock(R.RATEL_MAX_BLOCKS - 1, sizes, cuda_dev, wd_flags=[i % 2 for i in range(n_r)])
+    small = GpuBlock(0, [4096 * 3 + 1], cuda_dev)
+    run([big, small], 3)
+    with ratel_lib():
+        b = GpuBlock(5, [8] * (n_r + 1), cuda_dev)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_register_block(5, b.ranges(), R.RATEL_DEVICE)
+        assert e.value.code == R.RATEL_EINVAL
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_register_block(R.RATEL_MAX_BLOCKS, b.ranges()[:1], R.RATEL_DEVICE)
+        assert e.value.code == R.RATEL_EINVAL
+
+
+def test_clip_adam_l2_pinned_host(cuda_dev):
+    """Clip + Adam-L2 + pinned-host residency together, multi-range."""
+    blocks = [GpuBlock(i, [30_011 + i, 515], cuda_dev, pinned=True, wd_flags=[1, 0]) for i in range(3)]
+    run(blocks, 4, mode=oracle.ADAM_L2, max_norm=1e-3, tile_elems=4096)
