@@ -190,7 +190,8 @@ def workload_config(args, world):
     if args.blocks:
         sizes = sizes[:args.blocks]
     P = sum(sizes)
-    resid = "pinned-host" if args.residency == "host" else "device"
+    resid = {"host": "pinned-host", "hostcompute": "pinned-host, CPU handler (HOST_COMPUTE)"}.get(
+        args.residency, "device")
     name = {"13B": "13B", "30B": "30B", "70B": "70B (Table IV shape, 64.9B)", "175B": "175B",
             "c1": "C1 tiny block"}[shape]
     return {"workload": f"{name} GPT model states ({len(sizes)} blocks), {resid}-resident, AdamW, "
@@ -513,7 +514,8 @@ def main():
     ap.add_argument("--impl", default="ratel", choices=["ratel", "reference"])
     ap.add_argument("--shape", default="13B", choices=list(SHAPES))
     ap.add_argument("--blocks", type=int, default=0, help="use only the first N blocks")
-    ap.add_argument("--residency", default="device", choices=["device", "host"])
+    ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute"])
+    ap.add_argument("--host-threads", type=int, default=0)
     ap.add_argument("--clip", type=float, default=0.0)
     ap.add_argument("--max-ctas", type=int, default=0)
     ap.add_argument("--e2e-blocks", type=int, default=4)
@@ -566,11 +568,12 @@ def main():
         cfg.tile_elems = args.tile_elems
     if args.depth:
         cfg.pipeline_depth = args.depth
+    cfg.host_threads = args.host_threads
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
     try:
-        model = Model(R, torch, dev, sizes, world, rank, args.residency)
-        res = R.RATEL_PINNED_HOST if args.residency == "host" else R.RATEL_DEVICE
+        model = Model(R, torch, dev, sizes, world, rank, "device" if args.residency == "device" else "host")
+        res = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
         for b in range(len(sizes)):
             R.ratel_register_block(b, [model.ranges[b]], res)
         s = torch.cuda.Stream(device=dev)

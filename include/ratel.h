@@ -77,10 +77,23 @@ enum {
   RATEL_ENONFINITE = -6  /* clip mode: global grad norm was NaN/Inf (update still applied, like torch) */
 };
 
-typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1 } ratel_residency;
+/* Where a block's fp32 states live and who updates them:
+ *   DEVICE        states in HBM, the fused GPU kernel updates them in place;
+ *   PINNED_HOST   states in page-locked host memory, streamed H2D/D2H through
+ *                 a ring of device tiles around the same GPU kernel (the
+ *                 paper's Fig. 3b pipeline with the host link as the link);
+ *   HOST_COMPUTE  the paper's own design (§IV-C; CPU optimizer
+ *                 P:L582-584): states in page-locked host memory, G16 copied
+ *                 device->host (2 B/param), the CPU updates the states and
+ *                 produces P16 (double arithmetic, OpenMP), P16 copied
+ *                 host->device (2 B/param); stream-ordered via
+ *                 cudaLaunchHostFunc, the host thread never blocks. */
+typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2 } ratel_residency;
 typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
 /* Pinned-host staging schedule: PIPELINED = Fig. 3b (stage-in of tile k+1,
- * update of tile k and write-back of tile k-1 overlap on three streams);
+ * update of tile k and write-back of tile k-1 overlap on three streams; the
+ * tile updates run on a high-priority stream so they slot in between
+ * backward kernels);
  * SERIALIZED = Fig. 3a (naive AGO: stage-in, update, write-back in series). */
 typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1 } ratel_staging;
 
@@ -94,12 +107,13 @@ typedef enum { RATEL_COMM_AUTO = 0, RATEL_COMM_NONE = 1, RATEL_COMM_NCCL = 2 } r
 typedef struct {
   int mode;               /* ratel_mode; default RATEL_ADAMW */
   double max_grad_norm;   /* > 0 enables the global L2-norm clip (torch clip_grad_norm_); default 0 */
-  int pipeline_depth;     /* pinned-host tile ring depth, 2 or 3; default 3 */
+  int pipeline_depth;     /* pinned-host tile ring depth (slots of {theta,m,v} tiles), 2..16; default 4 */
   int staging;            /* ratel_staging; default PIPELINED */
   uint64_t tile_elems;    /* pinned-host tile length in elements, multiple of 8; default 1<<24 */
   int max_ctas;           /* cap on the update kernel's grid (0 = SMs x resident CTAs) */
   int timing;             /* 1: bracket every update-kernel launch with CUDA events (ratel_kernel_timing) */
   int comm;               /* ratel_comm; default RATEL_COMM_AUTO */
+  int host_threads;       /* HOST_COMPUTE handler threads (0 = OpenMP default: all cores) */
 } ratel_config;
 
 /* One contiguous parameter range of a block (a flat tensor, or a block's
@@ -146,8 +160,9 @@ int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id,
 /* Registers block `block_id` (0 <= id < RATEL_MAX_BLOCKS, each id once) made
  * of n_ranges (1..RATEL_MAX_RANGES_PER_BLOCK) ranges, all with the given
  * residency (ratel_residency).  Validates pointer kinds (device pointers on
- * this device; pinned host for RATEL_PINNED_HOST -- pageable memory is
- * RATEL_EINVAL), alignment and sizes.  The ranges array is copied.  Not
+ * this device; pinned host for RATEL_PINNED_HOST / RATEL_HOST_COMPUTE --
+ * pageable memory is RATEL_EINVAL), alignment and sizes.  HOST_COMPUTE blocks
+ * get library-owned pinned G16/P16 staging (4 B/param of the rank slice).  The ranges array is copied.  Not
  * allowed while a step is in flight (RATEL_ESTATE). */
 int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, int residency);
 

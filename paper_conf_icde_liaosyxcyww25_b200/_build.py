@@ -15,8 +15,8 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libratel.so")
-SOURCES = ["ratel_runtime.cu", "ratel_gen.cu"]
-HEADERS = ["ratel_kernels.cuh", "ratel_bf16.cuh", "nccl_dl.h"]
+SOURCES = ["ratel_runtime.cu", "ratel_gen.cu", "ratel_host_adam.cpp"]
+HEADERS = ["ratel_kernels.cuh", "ratel_bf16.cuh", "nccl_dl.h", "ratel_host_adam.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 
@@ -55,11 +55,11 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
     if out is None and not force and not stale():
         return LIB
     tmp = target + f".tmp{os.getpid()}"
-    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2",
+    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2,-fopenmp",
            *[f"-D{d}" for d in defines],
            "-Xptxas", "-v" if verbose else "-O3", "-shared", "-o", tmp,
            "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(),
-           *[os.path.join(CSRC, f) for f in SOURCES], "-ldl"]
+           *[os.path.join(CSRC, f) for f in SOURCES], "-ldl", "-lgomp"]
     r = subprocess.run(cmd, capture_output=True, text=True)
     if r.returncode != 0:
         sys.stderr.write(r.stdout + r.stderr)

@@ -24,6 +24,7 @@
 
 #include "nccl_dl.h"
 #include "ratel.h"
+#include "ratel_host_adam.h"
 #include "ratel_kernels.cuh"
 
 namespace {
@@ -40,6 +41,8 @@ int set_error(int code, const char* fmt, ...) {
   return code;
 }
 
+constexpr int kMaxDepth = 16;  // pinned-host tile ring slots
+
 struct Slice {
   uint64_t begin = 0, end = 0;
 };
@@ -51,8 +54,18 @@ struct Block {
   std::vector<ratel_range> ranges;
   std::vector<Slice> slices;
   cudaEvent_t ev_grad = nullptr;  // "gradient arrived" -- recorded on the caller's stream
-  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt
+  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt (s_host for HOST_COMPUTE)
+  cudaEvent_t ev_gh = nullptr;    // HOST_COMPUTE: G16 slices landed in host staging
+  std::vector<uint16_t*> h_g, h_p;  // HOST_COMPUTE: pinned G16 / P16 staging per range (rank slice)
   bool handed_off = false, enqueued = false;
+};
+
+// One host-handler invocation (owned by the callback, deleted when done).
+struct HostTask {
+  std::vector<HostAdamArgs> ranges;
+  const double* sumsq = nullptr;  // clip: pinned copy of the global sum of squares
+  double max_norm = 0.0;
+  int threads = 0;
 };
 
 struct TimingPair {
@@ -66,8 +79,12 @@ struct Ctx {
   int device = 0, rank = 0, world = 1;
   ratel_config cfg{};
   int sms = 0, k1_grid = 0, k2_grid = 0;
-  cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr;
-  cudaEvent_t ev_end[4] = {nullptr, nullptr, nullptr, nullptr};
+  cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr, s_host = nullptr,
+               s_tile = nullptr;
+  cudaEvent_t ev_end[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+  cudaEvent_t ev_norm = nullptr;  // clip: global norm final (on s_opt)
+  double* h_sumsq = nullptr;      // clip + HOST_COMPUTE: pinned copy of the norm
+  double hp_lr = 0, hp_b1 = 0, hp_b2 = 0, hp_eps = 0, hp_wd = 0, hp_bc1 = 1, hp_bc2 = 1;
   std::vector<Block> blocks;
   std::vector<int> reg;      // registered ids, registration order
   std::vector<int> pending;  // handed off before arming (deferred), hand-off order
@@ -83,7 +100,7 @@ struct Ctx {
   int* d_flag = nullptr;
   // pinned-host tile ring
   float* d_tiles = nullptr;  // depth x {theta, m, v} x tile
-  cudaEvent_t ev_h2d[3] = {}, ev_k1[3] = {}, ev_d2h[3] = {};
+  cudaEvent_t ev_h2d[kMaxDepth] = {}, ev_k1[kMaxDepth] = {}, ev_d2h[kMaxDepth] = {};
   uint64_t ring_k = 0;
   // NCCL
   ncclComm_t comm = nullptr;
@@ -158,7 +175,7 @@ const uint16_t* grad_ptr(const ratel_range& r, const Slice& s) {
 #endif
 
 template <int MODE, bool CLIP>
-void launch_k1(const UpdateParams& P, unsigned grid) {
+void launch_k1(const UpdateParams& P, unsigned grid, cudaStream_t st) {
 #if RATEL_K1_TMA
   (void)grid;
   uint64_t tiles = 0;
@@ -166,9 +183,9 @@ void launch_k1(const UpdateParams& P, unsigned grid) {
   uint64_t cap = static_cast<uint64_t>(G.sms) * RATEL_TMA_CTAS_PER_SM;
   if (G.cfg.max_ctas > 0) cap = std::min<uint64_t>(cap, static_cast<uint64_t>(G.cfg.max_ctas));
   const unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
-  adam_update_tma_kernel<MODE, CLIP><<<g, kTmaThreads, kTmaSmemBytes, G.s_opt>>>(P);
+  adam_update_tma_kernel<MODE, CLIP><<<g, kTmaThreads, kTmaSmemBytes, st>>>(P);
 #else
-  adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, G.s_opt>>>(P);
+  adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(P);
 #endif
 }
 
@@ -182,7 +199,7 @@ cudaError_t prepare_k1() {
 #endif
 }
 
-int launch_update(const RangeDesc* rd, int nr) {
+int launch_update(const RangeDesc* rd, int nr, cudaStream_t st) {
   if (nr == 0) return RATEL_OK;
   UpdateParams P{};
   uint64_t max8 = 0;
@@ -207,15 +224,15 @@ int launch_update(const RangeDesc* rd, int nr) {
       G.tpool.push_back(t);
     }
     tp = &G.tpool[G.tused++];
-    CK(cudaEventRecord(tp->a, G.s_opt));
+    CK(cudaEventRecord(tp->a, st));
   }
   if (G.cfg.mode == RATEL_ADAMW)
-    clip ? launch_k1<RATEL_ADAMW, true>(P, grid) : launch_k1<RATEL_ADAMW, false>(P, grid);
+    clip ? launch_k1<RATEL_ADAMW, true>(P, grid, st) : launch_k1<RATEL_ADAMW, false>(P, grid, st);
   else
-    clip ? launch_k1<RATEL_ADAM_L2, true>(P, grid) : launch_k1<RATEL_ADAM_L2, false>(P, grid);
+    clip ? launch_k1<RATEL_ADAM_L2, true>(P, grid, st) : launch_k1<RATEL_ADAM_L2, false>(P, grid, st);
   CK(cudaGetLastError());
   ++G.launches;
-  if (tp) CK(cudaEventRecord(tp->b, G.s_opt));
+  if (tp) CK(cudaEventRecord(tp->b, st));
   return RATEL_OK;
 }
 
@@ -254,8 +271,8 @@ int stage_tile(const ratel_range& r, const Slice& s, uint64_t off, uint64_t len)
   rd.n = len;
   rd.wd_on = r.apply_weight_decay != 0;
   const bool serial = G.cfg.staging == RATEL_STAGING_SERIALIZED;
-  cudaStream_t in = serial ? G.s_opt : G.s_h2d;
-  cudaStream_t out = serial ? G.s_opt : G.s_d2h;
+  cudaStream_t in = serial ? G.s_tile : G.s_h2d;
+  cudaStream_t out = serial ? G.s_tile : G.s_d2h;
   if (!serial && G.ring_k >= static_cast<uint64_t>(G.cfg.pipeline_depth))
     CK(cudaStreamWaitEvent(in, G.ev_d2h[k], 0));  // slot free: its previous write-back done
   CK(cudaMemcpyAsync(th, r.master + off, bytes, cudaMemcpyHostToDevice, in));
@@ -263,11 +280,11 @@ int stage_tile(const ratel_range& r, const Slice& s, uint64_t off, uint64_t len)
   CK(cudaMemcpyAsync(v, r.exp_avg_sq + off, bytes, cudaMemcpyHostToDevice, in));
   if (!serial) {
     CK(cudaEventRecord(G.ev_h2d[k], in));
-    CK(cudaStreamWaitEvent(G.s_opt, G.ev_h2d[k], 0));
+    CK(cudaStreamWaitEvent(G.s_tile, G.ev_h2d[k], 0));
   }
-  RK(launch_update(&rd, 1));
+  RK(launch_update(&rd, 1, G.s_tile));
   if (!serial) {
-    CK(cudaEventRecord(G.ev_k1[k], G.s_opt));
+    CK(cudaEventRecord(G.ev_k1[k], G.s_tile));
     CK(cudaStreamWaitEvent(out, G.ev_k1[k], 0));
   }
   CK(cudaMemcpyAsync(r.master + off, th, bytes, cudaMemcpyDeviceToHost, out));
@@ -287,6 +304,76 @@ int allgather_block(const Block& B) {
     NK(g_nccl.AllGather(p + s * G.rank, p, s, ncclBfloat16, G.comm, G.s_comm));
   }
   NK(g_nccl.GroupEnd());
+  return RATEL_OK;
+}
+
+void CUDART_CB host_adam_cb(void* arg) {
+  HostTask* t = static_cast<HostTask*>(arg);
+  double coef = 1.0;
+  if (t->sumsq != nullptr) {  // torch clip_grad_norm_: min(1, max/(||g||+1e-6)), NaN propagates
+    const double c = t->max_norm / (std::sqrt(*t->sumsq) + 1e-6);
+    coef = (c < 1.0 || std::isnan(c)) ? c : 1.0;
+  }
+  for (HostAdamArgs& a : t->ranges) {
+    a.coef = coef;
+    host_adam_range(a, t->threads);
+  }
+  delete t;
+}
+
+// The paper-literal handler: G16 device->host, CPU AdamW on the host states,
+// P16 host->device -- all stream-ordered (cudaLaunchHostFunc), no host blocking.
+int enqueue_host_compute(Block& B) {
+  CK(cudaStreamWaitEvent(G.s_d2h, B.ev_grad, 0));
+  HostTask* task = new HostTask();
+  task->threads = G.cfg.host_threads;
+  if (G.cfg.max_grad_norm > 0.0) {
+    task->sumsq = G.h_sumsq;
+    task->max_norm = G.cfg.max_grad_norm;
+  }
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const ratel_range& r = B.ranges[i];
+    const Slice& s = B.slices[i];
+    const uint64_t n = s.end - s.begin;
+    if (n == 0) continue;
+    if (cudaMemcpyAsync(B.h_g[i], grad_ptr(r, s), n * 2, cudaMemcpyDeviceToHost, G.s_d2h) != cudaSuccess) {
+      delete task;
+      return sticky_fail(RATEL_ECUDA, "G16 D2H failed: %s", cudaGetErrorString(cudaGetLastError()));
+    }
+    HostAdamArgs a{};
+    a.g = B.h_g[i];
+    a.th = r.master;
+    a.m = r.exp_avg;
+    a.v = r.exp_avg_sq;
+    a.p = B.h_p[i];
+    a.n = n;
+    a.wd_on = r.apply_weight_decay != 0;
+    a.mode = G.cfg.mode;
+    a.lr = G.hp_lr;
+    a.beta1 = G.hp_b1;
+    a.beta2 = G.hp_b2;
+    a.eps = G.hp_eps;
+    a.wd = G.hp_wd;
+    a.bc1 = G.hp_bc1;
+    a.bc2 = G.hp_bc2;
+    a.coef = 1.0;
+    task->ranges.push_back(a);
+  }
+  cudaError_t e = cudaEventRecord(B.ev_gh, G.s_d2h);
+  if (e == cudaSuccess) e = cudaStreamWaitEvent(G.s_host, B.ev_gh, 0);
+  if (e == cudaSuccess) e = cudaLaunchHostFunc(G.s_host, host_adam_cb, task);
+  if (e != cudaSuccess) {
+    delete task;
+    return sticky_fail(RATEL_ECUDA, "host handler enqueue failed: %s", cudaGetErrorString(e));
+  }
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const Slice& s = B.slices[i];
+    const uint64_t n = s.end - s.begin;
+    if (n == 0) continue;
+    CK(cudaMemcpyAsync(static_cast<uint16_t*>(B.ranges[i].param_bf16) + s.begin, B.h_p[i], n * 2,
+                       cudaMemcpyHostToDevice, G.s_host));
+  }
+  CK(cudaEventRecord(B.ev_done, G.s_host));
   return RATEL_OK;
 }
 
@@ -311,8 +398,12 @@ int enqueue_block(Block& B) {
       d.wd_on = r.apply_weight_decay != 0;
       d.pad_ = 0;
     }
-    RK(launch_update(rd, nr));
-  } else {
+    RK(launch_update(rd, nr, G.s_opt));
+  } else if (B.residency == RATEL_PINNED_HOST) {
+    // Tile updates run on a HIGH-priority stream: each is short and gates the
+    // copy pipeline, so when a backward GEMM frees SMs they must go first.
+    CK(cudaStreamWaitEvent(G.s_tile, B.ev_grad, 0));
+    if (G.cfg.max_grad_norm > 0.0) CK(cudaStreamWaitEvent(G.s_tile, G.ev_norm, 0));
     for (size_t i = 0; i < B.ranges.size(); ++i) {
       const Slice& s = B.slices[i];
       const uint64_t n = s.end - s.begin;
@@ -320,7 +411,14 @@ int enqueue_block(Block& B) {
         RK(stage_tile(B.ranges[i], s, off, std::min<uint64_t>(G.cfg.tile_elems, n - off)));
     }
   }
-  CK(cudaEventRecord(B.ev_done, G.s_opt));
+  if (B.residency == RATEL_HOST_COMPUTE)
+    RK(enqueue_host_compute(B));
+  else
+    CK(cudaEventRecord(B.ev_done, B.residency == RATEL_PINNED_HOST ? G.s_tile : G.s_opt));
+  // Keep ratel_optimizer_stream() ordered after every read of this block's
+  // grad (so grad.record_stream(ratel_optimizer_stream()) stays sufficient).
+  if (B.residency == RATEL_PINNED_HOST) CK(cudaStreamWaitEvent(G.s_opt, B.ev_done, 0));
+  if (B.residency == RATEL_HOST_COMPUTE) CK(cudaStreamWaitEvent(G.s_opt, B.ev_gh, 0));
   if (G.comm != nullptr) RK(allgather_block(B));
   B.enqueued = true;
   return RATEL_OK;
@@ -335,6 +433,12 @@ int finalize_clip() {
   ++G.launches;
   if (G.comm != nullptr)
     NK(g_nccl.AllReduce(G.d_sumsq, G.d_sumsq + 1, 1, ncclFloat64, ncclSum, G.comm, G.s_opt));
+  CK(cudaEventRecord(G.ev_norm, G.s_opt));  // the tile stream and the host handler wait on it
+  if (G.h_sumsq != nullptr) {  // some block runs the host handler: it needs the norm on the host
+    CK(cudaStreamWaitEvent(G.s_host, G.ev_norm, 0));
+    CK(cudaMemcpyAsync(G.h_sumsq, G.comm != nullptr ? G.d_sumsq + 1 : G.d_sumsq, sizeof(double),
+                       cudaMemcpyDeviceToHost, G.s_host));
+  }
   for (int id : G.reg) RK(enqueue_block(G.blocks[id]));
   G.pending.clear();
   return RATEL_OK;
@@ -364,13 +468,15 @@ int validate_config(const ratel_config& c) {
   if (c.mode != RATEL_ADAMW && c.mode != RATEL_ADAM_L2) return set_error(RATEL_EINVAL, "cfg.mode");
   if (!(c.max_grad_norm >= 0.0) || !std::isfinite(c.max_grad_norm))
     return set_error(RATEL_EINVAL, "cfg.max_grad_norm must be finite and >= 0");
-  if (c.pipeline_depth != 2 && c.pipeline_depth != 3) return set_error(RATEL_EINVAL, "cfg.pipeline_depth must be 2 or 3");
+  if (c.pipeline_depth < 2 || c.pipeline_depth > kMaxDepth)
+    return set_error(RATEL_EINVAL, "cfg.pipeline_depth must be in [2, %d]", kMaxDepth);
   if (c.staging != RATEL_STAGING_PIPELINED && c.staging != RATEL_STAGING_SERIALIZED)
     return set_error(RATEL_EINVAL, "cfg.staging");
   if (c.tile_elems == 0 || (c.tile_elems & 7u)) return set_error(RATEL_EINVAL, "cfg.tile_elems must be a positive multiple of 8");
   if (c.max_ctas < 0) return set_error(RATEL_EINVAL, "cfg.max_ctas must be >= 0");
   if (c.comm != RATEL_COMM_AUTO && c.comm != RATEL_COMM_NONE && c.comm != RATEL_COMM_NCCL)
     return set_error(RATEL_EINVAL, "cfg.comm");
+  if (c.host_threads < 0) return set_error(RATEL_EINVAL, "cfg.host_threads must be >= 0");
   return RATEL_OK;
 }
 
@@ -389,12 +495,15 @@ void destroy_all() {
     Block& B = G.blocks[id];
     if (B.ev_grad) cudaEventDestroy(B.ev_grad);
     if (B.ev_done) cudaEventDestroy(B.ev_done);
+    if (B.ev_gh) cudaEventDestroy(B.ev_gh);
+    for (uint16_t* p : B.h_g) cudaFreeHost(p);
+    for (uint16_t* p : B.h_p) cudaFreeHost(p);
   }
   for (TimingPair& t : G.tpool) {
     cudaEventDestroy(t.a);
     cudaEventDestroy(t.b);
   }
-  for (int k = 0; k < 3; ++k) {
+  for (int k = 0; k < kMaxDepth; ++k) {
     if (G.ev_h2d[k]) cudaEventDestroy(G.ev_h2d[k]);
     if (G.ev_k1[k]) cudaEventDestroy(G.ev_k1[k]);
     if (G.ev_d2h[k]) cudaEventDestroy(G.ev_d2h[k]);
@@ -405,8 +514,10 @@ void destroy_all() {
   if (G.d_partials) cudaFree(G.d_partials);
   if (G.d_sumsq) cudaFree(G.d_sumsq);
   if (G.h_flag) cudaFreeHost(G.h_flag);
+  if (G.h_sumsq) cudaFreeHost(G.h_sumsq);
+  if (G.ev_norm) cudaEventDestroy(G.ev_norm);
   if (G.comm) g_nccl.CommDestroy(G.comm);
-  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm})
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile})
     if (s) cudaStreamDestroy(s);
   G.~Ctx();
   new (&G) Ctx();
@@ -430,8 +541,11 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK(cudaStreamCreateWithPriority(&G.s_h2d, cudaStreamNonBlocking, greatest));
   CK(cudaStreamCreateWithPriority(&G.s_d2h, cudaStreamNonBlocking, greatest));
   CK(cudaStreamCreateWithPriority(&G.s_comm, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_host, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_tile, cudaStreamNonBlocking, greatest));
+  CK(cudaEventCreateWithFlags(&G.ev_norm, cudaEventDisableTiming));
   for (cudaEvent_t& ev : G.ev_end) CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
-  for (int k = 0; k < 3; ++k) {
+  for (int k = 0; k < kMaxDepth; ++k) {
     CK(cudaEventCreateWithFlags(&G.ev_h2d[k], cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&G.ev_k1[k], cudaEventDisableTiming));
     CK(cudaEventCreateWithFlags(&G.ev_d2h[k], cudaEventDisableTiming));
@@ -478,12 +592,13 @@ void ratel_default_config(ratel_config* cfg) {
   if (cfg == nullptr) return;
   cfg->mode = RATEL_ADAMW;
   cfg->max_grad_norm = 0.0;
-  cfg->pipeline_depth = 3;
+  cfg->pipeline_depth = 4;
   cfg->staging = RATEL_STAGING_PIPELINED;
   cfg->tile_elems = 1ull << 24;
   cfg->max_ctas = 0;
   cfg->timing = 0;
   cfg->comm = RATEL_COMM_AUTO;
+  cfg->host_threads = 0;
 }
 
 uint64_t ratel_padded_numel(uint64_t numel, int world_size) {
@@ -551,7 +666,7 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     return set_error(RATEL_EINVAL, "ratel_register_block: block %d already registered", block_id);
   if (ranges == nullptr || n_ranges < 1 || n_ranges > RATEL_MAX_RANGES_PER_BLOCK)
     return set_error(RATEL_EINVAL, "ratel_register_block: need 1..%d ranges", RATEL_MAX_RANGES_PER_BLOCK);
-  if (residency != RATEL_DEVICE && residency != RATEL_PINNED_HOST)
+  if (residency != RATEL_DEVICE && residency != RATEL_PINNED_HOST && residency != RATEL_HOST_COMPUTE)
     return set_error(RATEL_EINVAL, "ratel_register_block: bad residency %d", residency);
   std::vector<Slice> slices(n_ranges);
   for (int i = 0; i < n_ranges; ++i) {
@@ -569,7 +684,7 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     RK(check_ptr(r.param_bf16, true, "param_bf16", i));
     RK(check_ptr(r.grad_bf16, true, "grad_bf16", i));
     if (has) {
-      const bool dev = residency == RATEL_DEVICE;
+      const bool dev = residency == RATEL_DEVICE;  // PINNED_HOST and HOST_COMPUTE: page-locked host
       RK(check_ptr(r.master, dev, "master", i));
       RK(check_ptr(r.exp_avg, dev, "exp_avg", i));
       RK(check_ptr(r.exp_avg_sq, dev, "exp_avg_sq", i));
@@ -594,6 +709,20 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     }
   }
   Block& B = G.blocks[block_id];
+  if (residency == RATEL_HOST_COMPUTE) {
+    if (G.h_sumsq == nullptr) {
+      CK(cudaHostAlloc(&G.h_sumsq, sizeof(double), cudaHostAllocDefault));
+      *G.h_sumsq = 0.0;
+    }
+    B.h_g.assign(n_ranges, nullptr);
+    B.h_p.assign(n_ranges, nullptr);
+    for (int i = 0; i < n_ranges; ++i) {
+      const uint64_t n = std::max<uint64_t>(8, slices[i].end - slices[i].begin);
+      CK(cudaHostAlloc(&B.h_g[i], n * 2, cudaHostAllocDefault));
+      CK(cudaHostAlloc(&B.h_p[i], n * 2, cudaHostAllocDefault));
+    }
+    CK(cudaEventCreateWithFlags(&B.ev_gh, cudaEventDisableTiming));
+  }
   CK(cudaEventCreateWithFlags(&B.ev_grad, cudaEventDisableTiming));
   CK(cudaEventCreateWithFlags(&B.ev_done, cudaEventDisableTiming));
   B.ranges.assign(ranges, ranges + n_ranges);
@@ -629,13 +758,26 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
   s.decay = static_cast<float>(1.0 - lr * weight_decay);
   s.wd = static_cast<float>(weight_decay);
   s.wd_d = weight_decay;
+  G.hp_lr = lr;
+  G.hp_b1 = beta1;
+  G.hp_b2 = beta2;
+  G.hp_eps = eps;
+  G.hp_wd = weight_decay;
+  G.hp_bc1 = bc1;
+  G.hp_bc2 = bc2;
   G.armed = true;
   G.last_step = step;
   if (G.cfg.max_grad_norm > 0.0) {
     if (!G.reg.empty() && G.n_handed == static_cast<int>(G.reg.size())) RK(finalize_clip());
     return RATEL_OK;
   }
-  for (int id : G.pending) RK(enqueue_block(G.blocks[id]));  // deferred ("Ratel+ZeRO") order
+  // Deferred ("Ratel+ZeRO"): the optimizer stage starts after
+  // the whole backward -- every handler stream waits for every gradient
+  // handed off so far before any state moves (s_opt already waited on each).
+  if (!G.pending.empty())
+    for (cudaStream_t st : {G.s_h2d, G.s_d2h, G.s_host, G.s_tile})
+      for (int id : G.pending) CK(cudaStreamWaitEvent(st, G.blocks[id].ev_grad, 0));
+  for (int id : G.pending) RK(enqueue_block(G.blocks[id]));
   G.pending.clear();
   return RATEL_OK;
 }
@@ -681,20 +823,21 @@ int ratel_sync(void* stream) {
     if (G.n_handed != static_cast<int>(G.reg.size()))
       return set_error(RATEL_ESTATE, "ratel_sync: %d of %zu blocks handed off", G.n_handed, G.reg.size());
   }
-  cudaStream_t ss[4] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm};
-  for (int i = 0; i < 4; ++i) CK(cudaEventRecord(G.ev_end[i], ss[i]));
+  constexpr int NS = 6;
+  cudaStream_t ss[NS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile};
+  for (int i = 0; i < NS; ++i) CK(cudaEventRecord(G.ev_end[i], ss[i]));
   // Order the internal streams too: the next step's stage-in must not read
   // host states still being written back, and its K1 must not overwrite a
   // P16 slice the all-gather is still sending.
-  for (int i = 0; i < 4; ++i)
-    for (int j = 0; j < 4; ++j)
+  for (int i = 0; i < NS; ++i)
+    for (int j = 0; j < NS; ++j)
       if (i != j) CK(cudaStreamWaitEvent(ss[i], G.ev_end[j], 0));
   reset_step_state();
   if (stream != nullptr) {
-    for (int i = 0; i < 4; ++i) CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), G.ev_end[i], 0));
+    for (int i = 0; i < NS; ++i) CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), G.ev_end[i], 0));
     CK(cudaGetLastError());
   } else {
-    for (int i = 0; i < 4; ++i) CK(cudaEventSynchronize(G.ev_end[i]));
+    for (int i = 0; i < NS; ++i) CK(cudaEventSynchronize(G.ev_end[i]));
   }
   if (G.comm) {
     ncclResult_t ar = ncclSuccess;
@@ -712,7 +855,7 @@ int ratel_sync(void* stream) {
 int ratel_finalize(void) {
   if (!G.inited) return set_error(RATEL_ESTATE, "ratel_finalize: not initialised");
   cudaSetDevice(G.device);
-  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm})
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile})
     if (s) cudaStreamSynchronize(s);
   destroy_all();
   cudaGetLastError();

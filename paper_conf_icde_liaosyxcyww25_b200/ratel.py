@@ -26,6 +26,7 @@ RATEL_ENONFINITE = -6
 
 RATEL_DEVICE = 0
 RATEL_PINNED_HOST = 1
+RATEL_HOST_COMPUTE = 2
 RATEL_ADAMW = 0
 RATEL_ADAM_L2 = 1
 RATEL_STAGING_PIPELINED = 0
@@ -56,6 +57,7 @@ class ratel_config(ctypes.Structure):
         ("max_ctas", ctypes.c_int),
         ("timing", ctypes.c_int),
         ("comm", ctypes.c_int),
+        ("host_threads", ctypes.c_int),
     ]
 
 

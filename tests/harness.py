@@ -42,13 +42,14 @@ class GpuBlock:
     pinned host memory; P16 and grads on the device."""
 
     def __init__(self, block_id: int, sizes, device, pinned: bool = False, wd_flags=None,
-                 world: int = 1, rank: int = 0):
+                 world: int = 1, rank: int = 0, host_compute: bool = False):
         self.id = block_id
         self.sizes = list(sizes)
         self.offs = np.concatenate([[0], np.cumsum(self.sizes)]).astype(int)
         self.total = int(self.offs[-1])
         self.dev = device
-        self.pinned = pinned
+        self.pinned = pinned or host_compute
+        self.host_compute = host_compute
         self.wd = list(wd_flags) if wd_flags is not None else [1] * len(self.sizes)
         th0 = synth.theta0(self.total, block=block_id)
         self.p16, self.g16, self.master, self.m, self.v = [], [], [], [], []
@@ -61,7 +62,7 @@ class GpuBlock:
             ref = oracle.Range.fresh(t, self.wd[i])
             self.p16.append(p)
             self.g16.append(torch.zeros(cap, dtype=torch.bfloat16, device=device))
-            if pinned:
+            if self.pinned:
                 mk = lambda x: torch.from_numpy(np.ascontiguousarray(x)).pin_memory()
             else:
                 mk = lambda x: torch.from_numpy(np.ascontiguousarray(x)).to(device)
@@ -76,7 +77,8 @@ class GpuBlock:
 
     def register(self):
         R.ratel_register_block(self.id, self.ranges(),
-                               R.RATEL_PINNED_HOST if self.pinned else R.RATEL_DEVICE)
+                               R.RATEL_HOST_COMPUTE if self.host_compute else
+                               (R.RATEL_PINNED_HOST if self.pinned else R.RATEL_DEVICE))
 
     def grads_np(self, step: int):
         g = synth.grad16(self.total, step=step, block=self.id)

@@ -68,7 +68,7 @@ def test_init_without_gpu_fails_cleanly():
         R.ratel_init(0, 1, 2, None)  # world > 1 needs a unique id
     assert e.value.code == R.RATEL_EINVAL
     cfg = R.ratel_default_config()
-    cfg.pipeline_depth = 4
+    cfg.pipeline_depth = 17
     with pytest.raises(R.RatelError) as e:
         R.ratel_init(0, 0, 1, None, cfg)
     assert e.value.code == R.RATEL_EINVAL
@@ -76,8 +76,9 @@ def test_init_without_gpu_fails_cleanly():
 
 def test_default_config():
     c = R.ratel_default_config()
-    assert (c.mode, c.max_grad_norm, c.pipeline_depth, c.staging, c.tile_elems, c.max_ctas, c.timing, c.comm) == \
-        (R.RATEL_ADAMW, 0.0, 3, R.RATEL_STAGING_PIPELINED, 1 << 24, 0, 0, R.RATEL_COMM_AUTO)
+    assert (c.mode, c.max_grad_norm, c.pipeline_depth, c.staging, c.tile_elems, c.max_ctas, c.timing, c.comm,
+            c.host_threads) == \
+        (R.RATEL_ADAMW, 0.0, 4, R.RATEL_STAGING_PIPELINED, 1 << 24, 0, 0, R.RATEL_COMM_AUTO, 0)
 
 
 @pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
@@ -116,7 +117,7 @@ def test_generator_keys_match_synth():
 
 
 def test_struct_layouts_match_header():
-    # ratel_config: int, double, int, int, uint64, int, int, int -> 48 bytes
+    # ratel_config: int, double, int, int, uint64, int, int, int, int -> 48 bytes
     assert ctypes.sizeof(R.ratel_config) == 48
     assert R.ratel_config.tile_elems.offset == 24
     # ratel_range: 2 ptrs, int, 3 ptrs, uint64, int -> 64 bytes

@@ -448,3 +448,23 @@ def test_clip_adam_l2_pinned_host(cuda_dev):
     """Clip + Adam-L2 + pinned-host residency together, multi-range."""
     blocks = [GpuBlock(i, [30_011 + i, 515], cuda_dev, pinned=True, wd_flags=[1, 0]) for i in range(3)]
     run(blocks, 4, mode=oracle.ADAM_L2, max_norm=1e-3, tile_elems=4096)
+
+
+# ------------------------------------------- HOST_COMPUTE (the paper's CPU handler)
+@pytest.mark.parametrize("mode,max_norm", [(oracle.ADAMW, 0.0), (oracle.ADAM_L2, 0.0), (oracle.ADAMW, 1e-3)])
+def test_host_compute_vs_oracle(cuda_dev, mode, max_norm):
+    """RATEL_HOST_COMPUTE: G16 D2H, CPU AdamW in double on the pinned states,
+    P16 H2D (§IV-C) -- ragged multi-range blocks, 5 steps."""
+    blocks = [GpuBlock(0, [789_760 + 3, 256], cuda_dev, host_compute=True, wd_flags=[1, 0]),
+              GpuBlock(1, [65_537], cuda_dev, host_compute=True)]
+    run(blocks, 5, mode=mode, max_norm=max_norm, host_threads=4)
+
+
+def test_mixed_residencies_in_one_step(cuda_dev):
+    """Device, pinned-host and host-compute blocks handed off in one step,
+    AGO order and random order, with clipping across all of them."""
+    blocks = [GpuBlock(0, [100_003], cuda_dev),
+              GpuBlock(1, [70_001, 9], cuda_dev, pinned=True),
+              GpuBlock(2, [50_000], cuda_dev, host_compute=True),
+              GpuBlock(3, [12_345], cuda_dev)]
+    run(blocks, 3, order="random", max_norm=5e-3, tile_elems=8192)

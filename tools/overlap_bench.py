@@ -46,10 +46,11 @@ def run(args):
     cfg = R.ratel_default_config()
     cfg.timing = 1
     R.ratel_init(0, 0, 1, None, cfg)
-    model = bench.Model(R, torch, dev, sizes, 1, 0, args.residency, grad_ring=args.ring)
+    model = bench.Model(R, torch, dev, sizes, 1, 0, "device" if args.residency == "device" else "host",
+                        grad_ring=args.ring)
     R.ratel_finalize()
     ring = model.grad_ring
-    res_code = R.RATEL_PINNED_HOST if args.residency == "host" else R.RATEL_DEVICE
+    res_code = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
     vocab = bench.VOCAB if len(sizes) == L + 1 else 0
     hi = torch.cuda.Stream(priority=-2)
     order = list(reversed(range(len(sizes))))
@@ -59,7 +60,14 @@ def run(args):
         R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t_state["t"])
         t_state["t"] += 1
 
-    def one(schedule, bw):
+    side = torch.cuda.Stream()
+    tl = {}
+
+    def one(schedule, bw, timeline=False):
+        if timeline:
+            tl["t0"] = torch.cuda.Event(enable_timing=True)
+            tl["t0"].record(hi)
+            tl["g"], tl["d"] = {}, {}
         with torch.cuda.stream(hi):
             if schedule == "opt":
                 for b in order:
@@ -76,6 +84,13 @@ def run(args):
                         R.ratel_block_wait(b + args.ring, hi)   # ring slot free
                     bw.block(b, b % args.ring)
                     R.ratel_offload_grad_chunk(b, hi)
+                    if timeline:
+                        tl["g"][b] = torch.cuda.Event(enable_timing=True)
+                        tl["g"][b].record(hi)
+                        if schedule != "deferred":
+                            R.ratel_block_wait(b, side)
+                            tl["d"][b] = torch.cuda.Event(enable_timing=True)
+                            tl["d"][b].record(side)
                     if schedule == "naive" and args.residency == "device":
                         R.ratel_block_wait(b, hi)               # handler not overlapped
                 if schedule == "deferred":
@@ -117,6 +132,14 @@ def run(args):
                 sampler.mark(w0, time.time())
                 clk = sampler.stop() or {}
                 k1_ms, _ = R.ratel_kernel_timing(reset=True)
+                if args.timeline and sch in ("ago", "naive"):
+                    one(sch, bw, timeline=True)
+                    torch.cuda.synchronize()
+                    t0 = tl["t0"]
+                    print(json.dumps({"timeline": sch, "tokens": tokens,
+                                      "grad_ready_ms": {b: round(t0.elapsed_time(e), 1) for b, e in tl["g"].items()},
+                                      "update_done_ms": {b: round(t0.elapsed_time(e), 1) for b, e in tl["d"].items()}}),
+                          flush=True)
                 times[sch] = (e0.elapsed_time(e1) / args.steps, k1_ms / args.steps, clk.get("sm_mhz"),
                               clk.get("power_w"))
                 R.ratel_finalize()
@@ -143,11 +166,12 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--shape", default="13B")
     ap.add_argument("--blocks", type=int, default=0)
-    ap.add_argument("--residency", default="device", choices=["device", "host"])
+    ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute"])
     ap.add_argument("--tokens", type=int, nargs="+", default=[2048, 8192, 32768])
     ap.add_argument("--max-ctas", type=int, nargs="+", default=[0, 32])
     ap.add_argument("--schedules", nargs="+", default=["bwd", "opt", "ago", "deferred", "naive"])
     ap.add_argument("--ring", type=int, default=3)
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=1)
+    ap.add_argument("--timeline", action="store_true", help="per-block grad-ready / update-done times")
     run(ap.parse_args())
