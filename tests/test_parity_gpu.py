@@ -468,3 +468,43 @@ def test_mixed_residencies_in_one_step(cuda_dev):
               GpuBlock(2, [50_000], cuda_dev, host_compute=True),
               GpuBlock(3, [12_345], cuda_dev)]
     run(blocks, 3, order="random", max_norm=5e-3, tile_elems=8192)
+
+
+@pytest.mark.parametrize("residency", ["device", "pinned", "host_compute"])
+def test_grad_freed_after_record_stream_then_reused(cuda_dev, residency):
+    """The ownership contract of ratel.h: a grad tensor freed right after its
+    hand-off with grad.record_stream(ratel_optimizer_stream()) must not be
+    recycled by torch's caching allocator before the update has read it --
+    here the freed memory is immediately reallocated and overwritten."""
+    n = 1_000_003
+    b = GpuBlock(0, [n], cuda_dev, pinned=(residency == "pinned"), host_compute=(residency == "host_compute"))
+    opt_stream = None
+    with ratel_lib():
+        b.register()
+        opt_stream = torch.cuda.ExternalStream(R.ratel_optimizer_stream())
+        for t in (1, 2, 3):
+            g = b.grads_np(t)[0]
+            gt = torch.empty(R.ratel_padded_numel(n, 1), dtype=torch.bfloat16, device=cuda_dev)
+            gt[:n].copy_(u16_to_torch(g, cuda_dev))
+            rng = R.make_range(b.p16[0], gt, b.master[0], b.m[0], b.v[0], n)
+            # re-register the block's grad pointer each step (fresh tensor) --
+            # registration is only allowed between steps, so finalize/init
+            R.ratel_finalize()
+            R.ratel_init(0, 0, 1, None, R.ratel_default_config())
+            R.ratel_register_block(0, [rng], {"device": R.RATEL_DEVICE, "pinned": R.RATEL_PINNED_HOST,
+                                              "host_compute": R.RATEL_HOST_COMPUTE}[residency])
+            opt_stream = torch.cuda.ExternalStream(R.ratel_optimizer_stream())
+            torch.cuda.synchronize()
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            torch.cuda._sleep(2_000_000)                 # keep the current stream busy
+            R.ratel_offload_grad_chunk(0, torch.cuda.current_stream())
+            gt.record_stream(opt_stream)
+            del gt
+            junk = torch.empty(R.ratel_padded_numel(n, 1), dtype=torch.bfloat16, device=cuda_dev)
+            junk.fill_(float("nan"))                     # would poison the update if reused too early
+            R.ratel_sync(torch.cuda.current_stream())
+            torch.cuda.synchronize()
+            del junk
+            oracle.adam_range(b.oracle[0], g, oracle.hparams(step=t))
+            check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne, what=f"{residency} t{t}")
+        del opt_stream

@@ -1,9 +1,9 @@
 """Range-sharded (N > 1) path on ONE GPU.
 
 gpurun gives one GPU and NCCL refuses two ranks on one device, so:
-1. Two ranks are simulated in one process with two separately loaded copies
-   of libratel.so (independent library state), each `ratel_init(rank r,
-   world 2)` with RATEL_COMM_NONE; the test plays the bf16 all-gather (X2)
+1. N = 2, 4, 8 ranks are simulated in one process with N separately loaded
+   copies of libratel.so (independent library state), each `ratel_init(rank
+   r, world N)` with RATEL_COMM_NONE; the test plays the bf16 all-gather (X2)
    with device copies.  The gathered P16 and the concatenated fp32 slices
    must equal the single-rank run bit for bit (R16): this checks the C
    runtime's slicing, rank offsets of grad/param pointers, padding and the
@@ -45,12 +45,15 @@ def _single_rank(dev, steps, **cfg_kw):
     return blocks
 
 
-def test_two_ranks_simulated_bitwise_equals_single_rank(cuda_dev, tmp_path):
-    steps, world = 3, 2
+@pytest.mark.parametrize("world", [2, 4, 8])
+def test_ranks_simulated_bitwise_equal_single_rank(cuda_dev, tmp_path, world):
+    steps = 3
     ref = _single_rank(cuda_dev, steps)
-    lib_copy = tmp_path / "libratel_rank1.so"
-    shutil.copy(R.LIB_PATH, lib_copy)
-    libs = [R.lib(), R.load_library(str(lib_copy))]
+    libs = [R.lib()]
+    for r in range(1, world):
+        lib_copy = tmp_path / f"libratel_rank{r}.so"
+        shutil.copy(R.LIB_PATH, lib_copy)
+        libs.append(R.load_library(str(lib_copy)))
     ranks = [[GpuBlock(i, [n], cuda_dev, world=world, rank=r) for i, n in enumerate(SIZES)]
              for r in range(world)]
     for r, L in enumerate(libs):
