@@ -437,6 +437,7 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
     sizes = [block_params(h)] * n_blk
     cfg = R.ratel_default_config()
     cfg.timing = 0
+    cfg.pipeline_depth = args.e2e_depth
     init_lib(R, torch, dev_index, rank, world, cfg)
     try:
         model = Model(R, torch, dev, sizes, world, rank, "host", grad_ring=1)
@@ -497,6 +498,8 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
                "ms_per_step": ms / K, "steps": K, "params": P, "blocks": n_blk,
                "host_link_gbs": achieved, "host_link_peak_gbs": link["duplex"],
                "host_link_frac": achieved / link["duplex"], "host_link_probe": link,
+               "workload": f"{n_blk} of the {args.shape} model's blocks ({sizes[0]:,} params each), "
+                           "pinned-host states through the same C ABI",
                "path": "pinned-host states (tile ring depth %d, %d-elem tiles)" % (cfg.pipeline_depth,
                                                                                    cfg.tile_elems)}
         del model
@@ -520,6 +523,7 @@ def main():
     ap.add_argument("--max-ctas", type=int, default=0)
     ap.add_argument("--e2e-blocks", type=int, default=4)
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-depth", type=int, default=8)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--oracle-sample", type=int, default=1 << 25)
@@ -602,7 +606,7 @@ def main():
         achieved = k1_bytes / (k1_ms / 1e3) / 1e9 if k1_ms > 0 else None
         tpp = ncu_traffic_per_param()
         per_launch = own * args.steps / max(k1_n, 1)
-        roof = {"bound": "hbm", "kernel": "adam_update_kernel (K1)", "achieved": achieved, "peak": peak,
+        roof = {"bound": "hbm", "kernel": "adam_update_tma_kernel (K1)", "achieved": achieved, "peak": peak,
                 "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
                 "traffic": (tpp * per_launch) if tpp else None,
                 "algorithmic_bytes_per_launch": BYTES_PER_PARAM * per_launch,
