@@ -293,9 +293,14 @@ class SynthBackward:
             off += o * i
 
 
+SIM_COMM_NONE = False   # --sim-comm-none: N ranks on ONE GPU, gloo group, no NCCL (test mode)
+
+
 def init_lib(R, torch, dev_index, rank, world, cfg):
     uid = None
-    if world > 1:
+    if world > 1 and SIM_COMM_NONE:
+        cfg.comm = R.RATEL_COMM_NONE   # P16 slices are not exchanged: a plumbing test, not a result
+    elif world > 1:
         import torch.distributed as dist
         buf = torch.zeros(128, dtype=torch.uint8, device=f"cuda:{dev_index}")
         if rank == 0:
@@ -379,7 +384,7 @@ def max_over_ranks(torch, x, world, dev):
     if world == 1:
         return x
     import torch.distributed as dist
-    t = torch.tensor([x], dtype=torch.float64, device=dev)
+    t = torch.tensor([x], dtype=torch.float64, device=dev if dist.get_backend() == "nccl" else "cpu")
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
 
@@ -524,6 +529,8 @@ def main():
     ap.add_argument("--e2e-blocks", type=int, default=4)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-depth", type=int, default=8)
+    ap.add_argument("--sim-comm-none", action="store_true",
+                    help="test mode: N ranks may share one GPU; gloo process group, library without NCCL")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--oracle-sample", type=int, default=1 << 25)
@@ -554,11 +561,18 @@ def main():
 
     import torch
     import paper_conf_icde_liaosyxcyww25_b200 as R
+    global SIM_COMM_NONE
+    SIM_COMM_NONE = args.sim_comm_none
+    if SIM_COMM_NONE:
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if SIM_COMM_NONE:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     cfgd = workload_config(args, world)
     sizes = model_blocks(args.shape)
