@@ -197,15 +197,18 @@ def workload_config(args, world):
     return {"workload": f"{name} GPT model states ({len(sizes)} blocks), {resid}-resident, AdamW, "
                         f"per-block AGO hand-off" + (", clip" if args.clip > 0 else ""),
             "params": P, "blocks": len(sizes), "block_params": sizes[0], "residency": resid,
-            "parallelism": f"range-sharded x{world}" if world > 1 else "single GPU",
+            "parallelism": (f"range-sharded x{world}" + (" (fused peer-store all-gather)" if args.fused_allgather else
+                                                          " (NCCL all-gather)")) if world > 1 else "single GPU",
             "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
             "max_grad_norm": args.clip}
 
 
 class Model:
-    """Synthetic model states of one rank: per block one flat range."""
+    """Synthetic model states of one rank: per block one flat range.
+    symm=True allocates P16 in torch symmetric memory (peer-mapped) for the
+    fused update + all-gather (ratel_register_peer_params)."""
 
-    def __init__(self, R, torch, dev, sizes, world, rank, residency, grad_ring=2, pin_grads=False):
+    def __init__(self, R, torch, dev, sizes, world, rank, residency, grad_ring=2, pin_grads=False, symm=False):
         self.sizes = sizes
         self.ranges = []
         self.keep = []
@@ -216,11 +219,20 @@ class Model:
             key = R.ratel_gen_stream_key(0x5EED5EED, 2, 1, i)
             R.ratel_gen_grad16(g.data_ptr(), cap_max, 0, key)
         self.p16 = []
+        self.peer_ptrs = []
         for b, n in enumerate(sizes):
             cap = R.ratel_padded_numel(n, world)
             beg, end = R.ratel_rank_slice(n, world, rank)
             s = max(end - beg, 8)
-            p = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+            if symm:
+                import torch.distributed as dist
+                import torch.distributed._symmetric_memory as symm_mem
+                p = symm_mem.empty(cap, dtype=torch.bfloat16, device=dev)
+                p.zero_()
+                hdl = symm_mem.rendezvous(p, dist.group.WORLD.group_name)
+                self.peer_ptrs.append(list(hdl.buffer_ptrs))
+            else:
+                p = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
             if residency == "device":
                 th = torch.empty(s, dtype=torch.float32, device=dev)
                 m = torch.zeros(s, dtype=torch.float32, device=dev)
@@ -529,6 +541,8 @@ def main():
     ap.add_argument("--e2e-blocks", type=int, default=4)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--e2e-depth", type=int, default=8)
+    ap.add_argument("--fused-allgather", action="store_true",
+                    help="N>1: P16 in torch symmetric memory, all-gather fused into the update kernel")
     ap.add_argument("--sim-comm-none", action="store_true",
                     help="test mode: N ranks may share one GPU; gloo process group, library without NCCL")
     ap.add_argument("--no-e2e", action="store_true")
@@ -590,10 +604,14 @@ def main():
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
     try:
-        model = Model(R, torch, dev, sizes, world, rank, "device" if args.residency == "device" else "host")
+        fused = args.fused_allgather and world > 1 and not SIM_COMM_NONE
+        model = Model(R, torch, dev, sizes, world, rank, "device" if args.residency == "device" else "host",
+                      symm=fused)
         res = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
         for b in range(len(sizes)):
             R.ratel_register_block(b, [model.ranges[b]], res)
+            if fused:   # update kernel stores P16 into every peer over NVLink; no NCCL all-gather
+                R.ratel_register_peer_params(b, 0, model.peer_ptrs[b])
         s = torch.cuda.Stream(device=dev)
         order = list(reversed(range(len(sizes))))          # decreasing index
         t = 1

@@ -166,6 +166,18 @@ int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id,
  * allowed while a step is in flight (RATEL_ESTATE). */
 int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, int residency);
 
+/* Fused update + all-gather over peer memory (multi-GPU).  peer_params[q]
+ * (q = 0..world_size-1) is rank q's param_bf16 buffer of range `range_idx`
+ * of block `block_id`, as mapped into THIS process (CUDA IPC, P2P or
+ * torch.distributed._symmetric_memory buffer pointers); entry [rank] and
+ * NULL entries are skipped.  From then on the update kernel stores this
+ * rank's P16 slice of that range directly into every peer's buffer (NVLink
+ * P2P stores inside the kernel, overlapping the HBM streaming) and the NCCL
+ * all-gather of that range is skipped; ratel_sync adds one 8-byte allreduce
+ * as the cross-rank barrier.  Not for RATEL_HOST_COMPUTE blocks.  Between
+ * steps only.  The pointers are borrowed like all registered memory. */
+int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_params, int n);
+
 /* Arms optimizer step `step` (1-based t, strictly increasing across steps)
  * with the given hyperparameters (0 <= beta < 1, lr, eps, wd >= 0, finite).
  * Blocks already handed off in this step are enqueued now (deferred mode);

@@ -53,9 +53,20 @@ struct RangeDesc {
   int pad_;
 };
 
+// Fused all-gather over peer memory: this rank's P16 slice is also stored
+// straight into every other rank's P16 buffer (NVLink P2P stores) --
+// pointers already offset to the slice start of this range.
+constexpr int kMaxPeers = 8;
+struct PeerDesc {
+  uint16_t* p[kMaxPeers];
+  int n;
+};
+
 struct UpdateParams {
   RangeDesc r[kMaxRanges];
+  PeerDesc peers[kMaxRanges];
   int nr;
+  int any_peers;
   AdamScalars s;
   const double* sumsq;   // clip: global sum of g^2 (device); unused otherwise
   double max_norm;
@@ -171,6 +182,12 @@ __device__ __forceinline__ uint4 ld_g8(const uint16_t* p) {
 #endif
 }
 
+__device__ __forceinline__ void st_peers8(const PeerDesc& pd, uint64_t elem, uint4 v) {
+  for (int q = 0; q < pd.n; ++q)
+    asm volatile("st.global.v4.b32 [%0], {%1,%2,%3,%4};" ::"l"(pd.p[q] + elem), "r"(v.x), "r"(v.y),
+                 "r"(v.z), "r"(v.w) : "memory");
+}
+
 __device__ __forceinline__ void st_p8(uint16_t* p, uint4 v) {
 #if RATEL_K1_LDST == 2
   *reinterpret_cast<uint4*>(p) = v;
@@ -194,7 +211,8 @@ __device__ __forceinline__ void load8(Frag8& f, const RangeDesc& R, uint64_t i) 
 
 template <int MODE, bool CLIP>
 __device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint64_t i,
-                                              const AdamScalars& s, float coef_f, double coef_d) {
+                                              const AdamScalars& s, float coef_f, double coef_d,
+                                              const PeerDesc& pd) {
   const uint32_t gw[4] = {f.g.x, f.g.y, f.g.z, f.g.w};
   const bool wd = R.wd_on != 0;
 #pragma unroll
@@ -212,18 +230,21 @@ __device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint
   pk.z = pack_bf16x2_rn(f.t[4], f.t[5]);
   pk.w = pack_bf16x2_rn(f.t[6], f.t[7]);
   st_p8(R.p + 8 * i, pk);
+  st_peers8(pd, 8 * i, pk);
 }
 
 template <int MODE, bool CLIP>
 __device__ __forceinline__ void update_scalar(const RangeDesc& R, uint64_t j, const AdamScalars& s,
-                                              float coef_f, double coef_d) {
+                                              float coef_f, double coef_d, const PeerDesc& pd) {
   float g = bf16_bits_to_f32(R.g[j]);
   float th = R.th[j], m = R.m[j], v = R.v[j];
   adam_update<MODE, CLIP>(g, th, m, v, s, R.wd_on != 0, coef_f, coef_d);
   R.th[j] = th;
   R.m[j] = m;
   R.v[j] = v;
-  R.p[j] = static_cast<uint16_t>(pack_bf16x2_rn(th, 0.0f) & 0xFFFFu);
+  const uint16_t pb = static_cast<uint16_t>(pack_bf16x2_rn(th, 0.0f) & 0xFFFFu);
+  R.p[j] = pb;
+  for (int q = 0; q < pd.n; ++q) pd.p[q][j] = pb;
 }
 
 __device__ __forceinline__ double clip_coef_from(const double* sumsq, double max_norm, int* flag) {
@@ -253,16 +274,17 @@ __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(co
 #pragma unroll
       for (int u = 0; u < U; ++u) load8(f[u], R, i + u * stride);
 #pragma unroll
-      for (int u = 0; u < U; ++u) update_store8<MODE, CLIP>(f[u], R, i + u * stride, P.s, coef_f, coef_d);
+      for (int u = 0; u < U; ++u) update_store8<MODE, CLIP>(f[u], R, i + u * stride, P.s, coef_f, coef_d, P.peers[r]);
     }
     for (; i < n8; i += stride) {
       Frag8 f;
       load8(f, R, i);
-      update_store8<MODE, CLIP>(f, R, i, P.s, coef_f, coef_d);
+      update_store8<MODE, CLIP>(f, R, i, P.s, coef_f, coef_d, P.peers[r]);
     }
     const uint64_t j = (n8 << 3) + tid;
-    if (j < R.n) update_scalar<MODE, CLIP>(R, j, P.s, coef_f, coef_d);
+    if (j < R.n) update_scalar<MODE, CLIP>(R, j, P.s, coef_f, coef_d, P.peers[r]);
   }
+  if (P.any_peers) __threadfence_system();  // peer P16 stores visible before the step's barrier
 }
 
 // ---- K1, TMA-staged variant ------------------------------------------------
@@ -434,19 +456,19 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
 #if RATEL_TMA_RELEASE == 0
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // the stage's data is in registers now
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d, P.peers[t.r]);
 #elif RATEL_TMA_RELEASE == 1
       mbar_arrive(&empty[stage]);                 // every consumer thread arrives
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d, P.peers[t.r]);
 #elif RATEL_TMA_RELEASE == 2
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d, P.peers[t.r]);
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);  // after the values were consumed
 #elif RATEL_TMA_RELEASE == 3
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
       __syncwarp();
       if (lane == 0) mbar_arrive(&empty[stage]);
-      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d);
+      if (valid) update_store8<MODE, CLIP>(f, R, (t.off >> 3) + o, P.s, coef_f, coef_d, P.peers[t.r]);
 #else  // 4: results written back into the stage, bulk-stored by one thread
       if (valid) {
         const bool wd = R.wd_on != 0;
@@ -473,6 +495,7 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
         pk.z = pack_bf16x2_rn(f.t[4], f.t[5]);
         pk.w = pack_bf16x2_rn(f.t[6], f.t[7]);
         *reinterpret_cast<uint4*>(wb + 16 * o) = pk;
+        st_peers8(P.peers[t.r], t.off + 8 * o, pk);  // fused all-gather: NVLink P2P stores
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic smem writes -> async proxy
       asm volatile("bar.sync 1, %0;" ::"r"(kTmaConsumerWarps * 32) : "memory");
@@ -500,9 +523,10 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
     if (blockIdx.x == 0) {
       for (int r = 0; r < P.nr; ++r) {
         const uint64_t j = (P.r[r].n & ~7ull) + threadIdx.x;
-        if (j < P.r[r].n) update_scalar<MODE, CLIP>(P.r[r], j, P.s, coef_f, coef_d);
+        if (j < P.r[r].n) update_scalar<MODE, CLIP>(P.r[r], j, P.s, coef_f, coef_d, P.peers[r]);
       }
     }
+    if (P.any_peers) __threadfence_system();  // peer P16 stores visible before the step's barrier
   }
 }
 

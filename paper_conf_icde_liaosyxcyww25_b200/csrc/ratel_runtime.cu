@@ -57,6 +57,7 @@ struct Block {
   cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt (s_host for HOST_COMPUTE)
   cudaEvent_t ev_gh = nullptr;    // HOST_COMPUTE: G16 slices landed in host staging
   std::vector<uint16_t*> h_g, h_p;  // HOST_COMPUTE: pinned G16 / P16 staging per range (rank slice)
+  std::vector<std::vector<uint16_t*>> peers;  // per range: every rank's P16 base as mapped here (fused all-gather)
   bool handed_off = false, enqueued = false;
 };
 
@@ -95,7 +96,9 @@ struct Ctx {
   // clip
   double* d_partials = nullptr;
   size_t partial_cap = 0;  // slots
-  double* d_sumsq = nullptr;  // [0] this rank, [1] all ranks
+  double* d_sumsq = nullptr;  // [0] this rank, [1] all ranks, [2] barrier scratch
+  double* d_barrier = nullptr;
+  int n_peer_ranges = 0;      // ranges using the fused (peer-store) all-gather
   int* h_flag = nullptr;      // mapped pinned: non-finite norm seen
   int* d_flag = nullptr;
   // pinned-host tile ring
@@ -199,12 +202,16 @@ cudaError_t prepare_k1() {
 #endif
 }
 
-int launch_update(const RangeDesc* rd, int nr, cudaStream_t st) {
+int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* pd = nullptr) {
   if (nr == 0) return RATEL_OK;
   UpdateParams P{};
   uint64_t max8 = 0;
   for (int i = 0; i < nr; ++i) {
     P.r[i] = rd[i];
+    if (pd != nullptr) {
+      P.peers[i] = pd[i];
+      if (pd[i].n > 0) P.any_peers = 1;
+    }
     max8 = std::max<uint64_t>(max8, (rd[i].n + 7) / 8);
   }
   P.nr = nr;
@@ -254,8 +261,25 @@ int launch_sumsq(const Block& B) {
   return RATEL_OK;
 }
 
+// Peer P16 pointers of range i of B, offset to element `off` of this rank's
+// slice (empty when the range uses the NCCL all-gather).
+PeerDesc peer_desc(const Block& B, size_t i, uint64_t off) {
+  PeerDesc d{};
+  if (i < B.peers.size() && !B.peers[i].empty()) {
+    for (int q = 0; q < G.world; ++q) {
+      if (q == G.rank || B.peers[i][q] == nullptr) continue;
+      d.p[d.n++] = B.peers[i][q] + B.slices[i].begin + off;
+    }
+  }
+  return d;
+}
+
+bool has_peers(const Block& B, size_t i) { return i < B.peers.size() && !B.peers[i].empty(); }
+
 // One staged tile of a pinned-host range: H2D(theta, m, v) -> K1 -> D2H.
-int stage_tile(const ratel_range& r, const Slice& s, uint64_t off, uint64_t len) {
+int stage_tile(const Block& B, size_t ri, uint64_t off, uint64_t len) {
+  const ratel_range& r = B.ranges[ri];
+  const Slice& s = B.slices[ri];
   const int k = static_cast<int>(G.ring_k % static_cast<uint64_t>(G.cfg.pipeline_depth));
   const uint64_t T = G.cfg.tile_elems;
   float* th = G.d_tiles + (3ull * k + 0) * T;
@@ -282,7 +306,8 @@ int stage_tile(const ratel_range& r, const Slice& s, uint64_t off, uint64_t len)
     CK(cudaEventRecord(G.ev_h2d[k], in));
     CK(cudaStreamWaitEvent(G.s_tile, G.ev_h2d[k], 0));
   }
-  RK(launch_update(&rd, 1, G.s_tile));
+  const PeerDesc pd = peer_desc(B, ri, off);
+  RK(launch_update(&rd, 1, G.s_tile, &pd));
   if (!serial) {
     CK(cudaEventRecord(G.ev_k1[k], G.s_tile));
     CK(cudaStreamWaitEvent(out, G.ev_k1[k], 0));
@@ -296,9 +321,14 @@ int stage_tile(const ratel_range& r, const Slice& s, uint64_t off, uint64_t len)
 }
 
 int allgather_block(const Block& B) {
+  bool any = false;
+  for (size_t i = 0; i < B.ranges.size(); ++i) any = any || !has_peers(B, i);
+  if (!any) return RATEL_OK;  // every range is gathered by the update kernel's peer stores
   CK(cudaStreamWaitEvent(G.s_comm, B.ev_done, 0));
   NK(g_nccl.GroupStart());
-  for (const ratel_range& r : B.ranges) {
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    if (has_peers(B, i)) continue;
+    const ratel_range& r = B.ranges[i];
     const uint64_t s = padded(r.numel, G.world) / G.world;
     uint16_t* p = static_cast<uint16_t*>(r.param_bf16);
     NK(g_nccl.AllGather(p + s * G.rank, p, s, ncclBfloat16, G.comm, G.s_comm));
@@ -383,11 +413,13 @@ int enqueue_host_compute(Block& B) {
 int enqueue_block(Block& B) {
   if (B.residency == RATEL_DEVICE) {
     RangeDesc rd[kMaxRanges];
+    PeerDesc pd[kMaxRanges];
     int nr = 0;
     for (size_t i = 0; i < B.ranges.size(); ++i) {
       const ratel_range& r = B.ranges[i];
       const Slice& s = B.slices[i];
       if (s.end == s.begin) continue;
+      pd[nr] = peer_desc(B, i, 0);
       RangeDesc& d = rd[nr++];
       d.g = grad_ptr(r, s);
       d.th = r.master;
@@ -398,7 +430,7 @@ int enqueue_block(Block& B) {
       d.wd_on = r.apply_weight_decay != 0;
       d.pad_ = 0;
     }
-    RK(launch_update(rd, nr, G.s_opt));
+    RK(launch_update(rd, nr, G.s_opt, pd));
   } else if (B.residency == RATEL_PINNED_HOST) {
     // Tile updates run on a HIGH-priority stream: each is short and gates the
     // copy pipeline, so when a backward GEMM frees SMs they must go first.
@@ -408,7 +440,7 @@ int enqueue_block(Block& B) {
       const Slice& s = B.slices[i];
       const uint64_t n = s.end - s.begin;
       for (uint64_t off = 0; off < n; off += G.cfg.tile_elems)
-        RK(stage_tile(B.ranges[i], s, off, std::min<uint64_t>(G.cfg.tile_elems, n - off)));
+        RK(stage_tile(B, i, off, std::min<uint64_t>(G.cfg.tile_elems, n - off)));
     }
   }
   if (B.residency == RATEL_HOST_COMPUTE)
@@ -562,8 +594,9 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK((prepare_k1<RATEL_ADAM_L2, true>()));
   if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
   G.k2_grid = G.sms * 4;
-  CK(cudaMalloc(&G.d_sumsq, 2 * sizeof(double)));
-  CK(cudaMemset(G.d_sumsq, 0, 2 * sizeof(double)));
+  CK(cudaMalloc(&G.d_sumsq, 3 * sizeof(double)));
+  CK(cudaMemset(G.d_sumsq, 0, 3 * sizeof(double)));
+  G.d_barrier = G.d_sumsq + 2;
   CK(cudaHostAlloc(&G.h_flag, sizeof(int), cudaHostAllocMapped));
   *G.h_flag = 0;
   CK(cudaHostGetDevicePointer(reinterpret_cast<void**>(&G.d_flag), G.h_flag, 0));
@@ -734,6 +767,32 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
   return RATEL_OK;
 }
 
+int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_params, int n) {
+  RK(entry());
+  if (G.armed || G.n_handed > 0) return set_error(RATEL_ESTATE, "ratel_register_peer_params: a step is in flight");
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_params: block %d is not registered", block_id);
+  Block& B = G.blocks[block_id];
+  if (range_idx < 0 || range_idx >= static_cast<int>(B.ranges.size()))
+    return set_error(RATEL_EINVAL, "ratel_register_peer_params: range %d out of range", range_idx);
+  if (B.residency == RATEL_HOST_COMPUTE)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_params: HOST_COMPUTE blocks use the NCCL all-gather");
+  if (peer_params == nullptr || n != G.world || G.world - 1 > kMaxPeers)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_params: need world_size (%d <= %d) pointers", G.world,
+                     kMaxPeers + 1);
+  std::vector<uint16_t*> v(n, nullptr);
+  for (int q = 0; q < n; ++q) {
+    if (q == G.rank || peer_params[q] == nullptr) continue;
+    if (!aligned16(peer_params[q]))
+      return set_error(RATEL_EINVAL, "ratel_register_peer_params: peer pointers must be 16-byte aligned");
+    v[q] = static_cast<uint16_t*>(peer_params[q]);
+  }
+  if (B.peers.size() != B.ranges.size()) B.peers.resize(B.ranges.size());
+  if (B.peers[range_idx].empty()) ++G.n_peer_ranges;
+  B.peers[range_idx] = v;
+  return RATEL_OK;
+}
+
 int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay, int64_t step) {
   RK(entry());
   if (G.armed) return set_error(RATEL_ESTATE, "ratel_adam_step: step %lld already armed", (long long)G.last_step);
@@ -822,6 +881,17 @@ int ratel_sync(void* stream) {
     if (!G.armed) return set_error(RATEL_ESTATE, "ratel_sync: blocks handed off but no ratel_adam_step");
     if (G.n_handed != static_cast<int>(G.reg.size()))
       return set_error(RATEL_ESTATE, "ratel_sync: %d of %zu blocks handed off", G.n_handed, G.reg.size());
+  }
+  if (G.comm != nullptr && G.n_peer_ranges > 0) {
+    // Fused all-gather: ranks wrote into each other's P16.  One 8-byte
+    // allreduce after every local update is the cross-rank barrier: once it
+    // completes here, every rank's update kernels (and their peer stores,
+    // fenced system-wide) have finished.
+    CK(cudaEventRecord(G.ev_end[0], G.s_opt));
+    CK(cudaEventRecord(G.ev_end[5], G.s_tile));
+    CK(cudaStreamWaitEvent(G.s_comm, G.ev_end[0], 0));
+    CK(cudaStreamWaitEvent(G.s_comm, G.ev_end[5], 0));
+    NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
   }
   constexpr int NS = 6;
   cudaStream_t ss[NS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile};

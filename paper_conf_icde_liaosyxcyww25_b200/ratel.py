@@ -91,6 +91,7 @@ def load_library(path: str = _LIB_PATH):
         "ratel_offload_grad_chunk": (I, [I, P]),
         "ratel_sync": (I, [P]),
         "ratel_block_wait": (I, [I, P]),
+        "ratel_register_peer_params": (I, [I, I, ctypes.POINTER(P), I]),
         "ratel_finalize": (I, []),
         "ratel_last_error": (ctypes.c_char_p, []),
         "ratel_padded_numel": (U64, [U64, I]),
@@ -160,6 +161,13 @@ def ratel_init(device: int, rank: int = 0, world_size: int = 1, nccl_unique_id: 
 def ratel_register_block(block_id: int, ranges, residency: int = RATEL_DEVICE) -> None:
     arr = (ratel_range * len(ranges))(*ranges)
     _check(_lib.ratel_register_block(block_id, arr, len(ranges), residency))
+
+
+def ratel_register_peer_params(block_id: int, range_idx: int, peer_params) -> None:
+    """peer_params: one pointer (int, tensor or None) per rank."""
+    ptrs = [(p.data_ptr() if hasattr(p, "data_ptr") else (int(p) if p else None)) for p in peer_params]
+    arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
+    _check(_lib.ratel_register_peer_params(block_id, range_idx, arr, len(ptrs)))
 
 
 def ratel_adam_step(lr: float, beta1: float, beta2: float, eps: float, weight_decay: float, step: int) -> None:
