@@ -74,7 +74,7 @@ class ratel_range(ctypes.Structure):
     ]
 
 
-def load_library(path: str = _LIB_PATH):
+def load_library(path: str = _LIB_PATH, strict: bool = True):
     """Load a libratel.so build and declare its signatures (tools load
     build-variant copies through this; the package uses the in-tree one)."""
     if not os.path.exists(path):
@@ -107,6 +107,8 @@ def load_library(path: str = _LIB_PATH):
         "ratel_test_fill_f32": (I, [P, U64, ctypes.c_float, P]),
     }
     for name, (res, args) in sig.items():
+        if not strict and not hasattr(lib, name):
+            continue   # an older build variant (tools/ only)
         f = getattr(lib, name)
         f.restype = res
         f.argtypes = args
