@@ -508,3 +508,35 @@ def test_grad_freed_after_record_stream_then_reused(cuda_dev, residency):
             oracle.adam_range(b.oracle[0], g, oracle.hparams(step=t))
             check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne, what=f"{residency} t{t}")
         del opt_stream
+
+
+def test_back_to_back_steps_without_host_sync(cuda_dev):
+    """Five steps enqueued back to back with only stream-ordered syncs
+    (ratel_sync(stream)) -- grads rewritten on that stream each step -- over
+    device, pinned-host and host-compute blocks: cross-step ordering of the
+    library's internal streams, tile ring and host staging."""
+    blocks = [GpuBlock(0, [200_003], cuda_dev),
+              GpuBlock(1, [150_001], cuda_dev, pinned=True),
+              GpuBlock(2, [90_000, 13], cuda_dev, host_compute=True)]
+    steps = 5
+    host_grads = {t: {b.id: [u16_to_torch(g, "cpu").pin_memory() for g in b.grads_np(t)] for b in blocks}
+                  for t in range(1, steps + 1)}
+    s = torch.cuda.Stream()
+    with ratel_lib(tile_elems=16_384, pipeline_depth=2):
+        for b in blocks:
+            b.register()
+        torch.cuda.synchronize()
+        with torch.cuda.stream(s):
+            for t in range(1, steps + 1):
+                R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+                for b in reversed(blocks):
+                    for i, hg in enumerate(host_grads[t][b.id]):
+                        b.g16[i][:hg.numel()].copy_(hg, non_blocking=True)
+                    R.ratel_offload_grad_chunk(b.id, s)
+                R.ratel_sync(s)
+        s.synchronize()
+        for t in range(1, steps + 1):
+            oracle_step(blocks, t, {b.id: b.grads_np(t) for b in blocks})
+        for b in blocks:
+            for i in range(len(b.sizes)):
+                check_range(b.gpu_state(i), b.oracle[i], own_rne=oracle.bf16_rne, what=f"b{b.id} r{i}")
