@@ -109,6 +109,10 @@ def run(args):
     for tokens in args.tokens:
         bw = SynthBackward(dev, h, tokens, model.p16, ring, vocab)
         for mc in args.max_ctas:
+            # cuBLAS SM carve-out: the backward GEMMs size their grids for
+            # SMs - mc, leaving mc SMs to the update kernel (max_ctas = mc)
+            if args.carveout:
+                torch._C._set_sm_carveout_experimental(mc if mc > 0 else None)
             times = {}
             for sch in args.schedules:
                 if sch == "deferred" and args.ring < len(sizes):
@@ -144,7 +148,8 @@ def run(args):
                               clk.get("power_w"))
                 R.ratel_finalize()
             tb = times["bwd"][0]
-            row = {"residency": args.residency, "tokens": tokens, "max_ctas": mc, "blocks": len(sizes),
+            row = {"residency": args.residency, "tokens": tokens, "max_ctas": mc, "carveout": bool(args.carveout),
+                   "blocks": len(sizes),
                    "params": sum(sizes), "bwd_ms": tb, "bwd_tflops": 4 * sum(sizes) * tokens / (tb / 1e3) / 1e12}
             for sch, v in times.items():
                 row[f"{sch}_sm_mhz"], row[f"{sch}_power_w"] = v[2], v[3]
@@ -174,4 +179,5 @@ if __name__ == "__main__":
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=1)
     ap.add_argument("--timeline", action="store_true", help="per-block grad-ready / update-done times")
+    ap.add_argument("--carveout", action="store_true", help="cuBLAS SM carve-out = max_ctas for the backward")
     run(ap.parse_args())
