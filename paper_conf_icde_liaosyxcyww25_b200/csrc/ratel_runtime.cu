@@ -22,6 +22,8 @@
 #include <cstring>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "nccl_dl.h"
 #include "ratel.h"
 #include "ratel_host_adam.h"
@@ -32,6 +34,20 @@ namespace {
 using namespace ratel;
 
 thread_local char t_err[1024] = "";
+
+// NVTX ranges around the API calls, tile stages and host handlers (header-only
+// nvtx3: free unless a profiler is attached; nsys/ncu show the AGO schedule).
+struct Nvtx {
+  explicit Nvtx(const char* fmt, ...) {
+    char buf[96];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    nvtxRangePushA(buf);
+  }
+  ~Nvtx() { nvtxRangePop(); }
+};
 
 int set_error(int code, const char* fmt, ...) {
   va_list ap;
@@ -278,6 +294,7 @@ bool has_peers(const Block& B, size_t i) { return i < B.peers.size() && !B.peers
 
 // One staged tile of a pinned-host range: H2D(theta, m, v) -> K1 -> D2H.
 int stage_tile(const Block& B, size_t ri, uint64_t off, uint64_t len) {
+  Nvtx nv("ratel tile %llu", static_cast<unsigned long long>(G.ring_k));
   const ratel_range& r = B.ranges[ri];
   const Slice& s = B.slices[ri];
   const int k = static_cast<int>(G.ring_k % static_cast<uint64_t>(G.cfg.pipeline_depth));
@@ -339,6 +356,7 @@ int allgather_block(const Block& B) {
 
 void CUDART_CB host_adam_cb(void* arg) {
   HostTask* t = static_cast<HostTask*>(arg);
+  Nvtx nv("ratel host handler (%zu ranges)", t->ranges.size());
   double coef = 1.0;
   if (t->sumsq != nullptr) {  // torch clip_grad_norm_: min(1, max/(||g||+1e-6)), NaN propagates
     const double c = t->max_norm / (std::sqrt(*t->sumsq) + 1e-6);
@@ -794,6 +812,7 @@ int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_pa
 }
 
 int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay, int64_t step) {
+  Nvtx nv("ratel_adam_step %lld", static_cast<long long>(step));
   RK(entry());
   if (G.armed) return set_error(RATEL_ESTATE, "ratel_adam_step: step %lld already armed", (long long)G.last_step);
   if (step <= G.last_step)
@@ -842,6 +861,7 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
 }
 
 int ratel_offload_grad_chunk(int block_id, void* stream) {
+  Nvtx nv("ratel_offload_grad_chunk %d", block_id);
   RK(entry());
   if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
     return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d is not registered", block_id);
@@ -876,6 +896,7 @@ int ratel_block_wait(int block_id, void* stream) {
 }
 
 int ratel_sync(void* stream) {
+  Nvtx nv("ratel_sync");
   RK(entry());
   if (G.armed || G.n_handed > 0) {
     if (!G.armed) return set_error(RATEL_ESTATE, "ratel_sync: blocks handed off but no ratel_adam_step");

@@ -540,3 +540,34 @@ def test_back_to_back_steps_without_host_sync(cuda_dev):
         for b in blocks:
             for i in range(len(b.sizes)):
                 check_range(b.gpu_state(i), b.oracle[i], own_rne=oracle.bf16_rne, what=f"b{b.id} r{i}")
+
+
+def test_checkpoint_resume_bitwise(cuda_dev):
+    """Checkpoint/resume: states are caller-owned tensors.  Ten continuous
+    steps == five steps, copy P32/m/v/P16 out (torch.save-able), finalize,
+    re-init, register the restored copies and continue at t = 6..10."""
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 10, check_every=False)
+    b = _fresh(SIZES, cuda_dev)
+    run(b, 5, check_every=False)
+    ckpt = [[(x.clone(), y.clone(), z.clone(), p.clone()) for x, y, z, p in zip(bl.master, bl.m, bl.v, bl.p16)]
+            for bl in b]
+    c = _fresh(SIZES, cuda_dev)
+    for bl, saved in zip(c, ckpt):
+        for i, (x, y, z, p) in enumerate(saved):
+            bl.master[i].copy_(x)
+            bl.m[i].copy_(y)
+            bl.v[i].copy_(z)
+            bl.p16[i].copy_(p)
+    with ratel_lib():
+        for bl in c:
+            bl.register()
+        for t in range(6, 11):
+            for bl in c:
+                bl.load_grads(t)
+            torch.cuda.synchronize()
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            for bl in reversed(c):
+                R.ratel_offload_grad_chunk(bl.id, None)
+            R.ratel_sync(None)
+    assert_bitwise(snapshot(a), snapshot(c))
