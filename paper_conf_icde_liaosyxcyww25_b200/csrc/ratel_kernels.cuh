@@ -80,6 +80,9 @@ struct SumsqParams {
   double* partials;  // one slot per CTA
 };
 
+#ifndef RATEL_K1_NOMATH
+#define RATEL_K1_NOMATH 0
+#endif
 #ifndef RATEL_K1_FASTMATH
 #define RATEL_K1_FASTMATH 1
 #endif
@@ -477,7 +480,11 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
         for (int kk = 0; kk < 8; ++kk) {
           const uint32_t w = gw[kk >> 1];
           float g = bf16_bits_to_f32((kk & 1) ? (w >> 16) : (w & 0xFFFFu));
+#if RATEL_K1_NOMATH  // diagnostic build only: pure data movement through the same pipeline
+          f.t[kk] += g * 0.0f;
+#else
           adam_update<MODE, CLIP>(g, f.t[kk], f.m[kk], f.v[kk], P.s, wd, coef_f, coef_d);
+#endif
         }
         uint8_t* wb = smem + stage * kTmaStageBytes;
         float4* th = reinterpret_cast<float4*>(wb + kTmaTile * 2) + 2 * o;
