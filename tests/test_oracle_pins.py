@@ -284,3 +284,17 @@ def test_bf16_rne_exhaustive_vs_torch():
             bad = np.flatnonzero(mine != ref)[0]
             raise AssertionError(f"pattern {u[bad]:#010x}: {mine[bad]:#06x} vs {ref[bad]:#06x}")
         assert np.all((mine[isn] & 0x7FFF) > 0x7F80)
+
+
+def test_oracle_regression_digests():
+    """The oracle's C1 outputs are unchanged since tests/golden/ was written
+    (tests/golden/make_golden.py; regenerate only with a cited reason)."""
+    import json
+    import os
+    import importlib.util
+    here = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+    spec = importlib.util.spec_from_file_location("make_golden", os.path.join(here, "make_golden.py"))
+    mg = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(mg)
+    want = json.load(open(os.path.join(here, "oracle_digests.json")))["sha256"]
+    assert mg.digests() == want
