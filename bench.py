@@ -105,6 +105,8 @@ class ClockSampler:
     def mark(self, t0, t1):
         self.window = (t0, t1)
 
+    BAD = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown")
+
     def stop(self):
         if self.p is None:
             return None
@@ -114,7 +116,13 @@ class ClockSampler:
             self.p.wait(timeout=5)
         except Exception:
             self.p.kill()
-        t0, t1 = self.window or (0, 1e30)
+        return self.stats()
+
+    def stats(self, window=None):
+        """Clock summary of the samples inside `window` (default: the marked one)."""
+        if self.p is None:
+            return None
+        t0, t1 = window or self.window or (0, 1e30)
         rows = [r for (t, r) in self.samples if t0 - 0.05 <= t <= t1 + 0.15 and len(r) >= 7]
         if not rows:
             rows = [r for (_, r) in self.samples if len(r) >= 7][-3:]
@@ -619,15 +627,34 @@ def main():
             step_once(R, t, order, s)
             t += 1
         barrier(torch, world)
-        R.ratel_kernel_timing(reset=True)
-        l0 = R.ratel_launch_count()
-        w0 = time.time()
-        ms = timed_steps(R, torch, order, s, t, args.steps)
-        w1 = time.time()
-        launches = R.ratel_launch_count() - l0
-        k1_ms, k1_n = R.ratel_kernel_timing(reset=True)
-        if sampler:
-            sampler.mark(w0, w1)
+        remeasured = False
+        for attempt in range(2):
+            R.ratel_kernel_timing(reset=True)
+            l0 = R.ratel_launch_count()
+            w0 = time.time()
+            ms = timed_steps(R, torch, order, s, t, args.steps)
+            t += args.steps
+            w1 = time.time()
+            launches = R.ratel_launch_count() - l0
+            k1_ms, k1_n = R.ratel_kernel_timing(reset=True)
+            bad = 0.0
+            if sampler:
+                sampler.mark(w0, w1)
+                time.sleep(0.3)   # let the sampler deliver the window's last rows
+                st = sampler.stats() or {}
+                bad = 1.0 if any(r in ClockSampler.BAD for r in st.get("reasons", [])) else 0.0
+                if st.get("sm_mhz") and st.get("sm_max_mhz") and not st.get("reasons") \
+                        and st["sm_mhz"] < 0.6 * st["sm_max_mhz"]:
+                    bad = 1.0     # clocks stuck low with no reason: a leftover clock lock
+            if world > 1:        # every rank re-measures together
+                import torch.distributed as dist
+                flag = torch.tensor([bad], dtype=torch.float64,
+                                    device=dev if dist.get_backend() == "nccl" else "cpu")
+                dist.all_reduce(flag, op=dist.ReduceOp.MAX)
+                bad = float(flag.item())
+            if bad == 0.0 or attempt == 1:
+                break
+            remeasured = True     # throttled window (hw/thermal slowdown): measure once more
         ms = max_over_ranks(torch, ms, world, dev)
         barrier(torch, world)
         own = sum(e - b for (b, e) in model.slices)
@@ -648,7 +675,7 @@ def main():
         overlap = None
         if args.overlap_tokens > 0 and world == 1 and args.residency == "device" and args.clip == 0:
             try:
-                o, t = overlap_probe(args, R, torch, dev, model, sizes, order, t + args.steps)
+                o, t = overlap_probe(args, R, torch, dev, model, sizes, order, t)
                 opt_ms = ms / args.steps
                 overlap = {"tokens": args.overlap_tokens, "backward_ms": o["bwd"], "ago_step_ms": o["ago"],
                            "optimizer_alone_ms": opt_ms, "exposed_optimizer_ms": o["ago"] - o["bwd"],
@@ -685,7 +712,8 @@ def main():
                     "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
                     "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                     "config": cfgd, "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
-                    "clocks": clocks, "gpu_launches": launches, "overlap": overlap,
+                    "clocks": dict(clocks or {}, remeasured=remeasured), "gpu_launches": launches,
+                    "overlap": overlap,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
             print(json.dumps(line), flush=True)
     finally:
