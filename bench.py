@@ -418,6 +418,61 @@ def barrier(torch, world):
 
 
 # ------------------------------------------------------------------- e2e
+def run_e2e_device(args, R, torch, dev, model, sizes, order, t, world):
+    """e2e on the SAME workload as `value`: every step the gradients come
+    from pinned host memory (H2D before each block's hand-off) and the
+    updated P16 goes back to pinned host memory (D2H as soon as each block's
+    update ran), through the C ABI; the states stay resident."""
+    ring = model.grad_ring
+    nr = len(ring)
+    g_host = torch.empty(ring[0].numel(), dtype=torch.bfloat16, pin_memory=True)
+    g_host.copy_(ring[0])
+    p_host = [torch.empty(e - b, dtype=torch.bfloat16, pin_memory=True) for (b, e) in model.slices]
+    s_in = torch.cuda.Stream(device=dev)
+    s_out = torch.cuda.Stream(device=dev)
+    tt = [t]
+
+    def one():
+        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], tt[0])
+        tt[0] += 1
+        with torch.cuda.stream(s_in):
+            for j, b in enumerate(order):
+                if j >= nr:
+                    R.ratel_block_wait(order[j - nr], s_in)   # ring slot consumed
+                beg, end = model.slices[b]
+                ring[b % nr][beg:end].copy_(g_host[beg:end], non_blocking=True)   # G16 host -> device
+                R.ratel_offload_grad_chunk(b, s_in)
+        with torch.cuda.stream(s_out):
+            for b in order:
+                R.ratel_block_wait(b, s_out)
+                beg, end = model.slices[b]
+                p_host[b].copy_(model.p16[b][beg:end], non_blocking=True)      # P16 device -> host
+        s_in.wait_stream(s_out)
+        R.ratel_sync(s_in)
+
+    one()
+    barrier(torch, world)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    K = args.e2e_steps
+    e0.record(s_in)
+    for _ in range(K):
+        one()
+    e1.record(s_in)
+    e1.synchronize()
+    ms = max_over_ranks(torch, e0.elapsed_time(e1), world, dev)
+    own = sum(e - b for (b, e) in model.slices)
+    P = sum(sizes)
+    link = host_link_probe(torch, dev)
+    moved = 4 * own   # 2 B/param in, 2 B/param out, this rank
+    achieved = moved / (ms / K / 1e3) / 1e9
+    return {"value": P * K / (ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(2 * own * world),
+            "d2h_bytes_per_step": int(2 * own * world), "ms_per_step": ms / K, "steps": K,
+            "workload": "the value's workload (all blocks, states resident); G16 in from pinned host, "
+                        "P16 out to pinned host, every step",
+            "host_link_gbs": achieved, "host_link_peak_gbs": link["duplex"],
+            "host_link_frac": achieved / link["duplex"], "host_link_probe": link}, tt[0]
+
+
 def host_link_probe(torch, dev, nbytes=1 << 30, reps=3):
     """Measured duplex host-link bandwidth on this box (pinned H2D and D2H
     concurrently on two streams): the e2e roofline denominator."""
@@ -684,19 +739,28 @@ def main():
                            "grad_ring": len(model.grad_ring)}
             except Exception as ex:
                 overlap = {"error": repr(ex)[:300]}
+        e2e = None
+        if not args.no_e2e and args.residency == "device":
+            try:
+                e2e, t = run_e2e_device(args, R, torch, dev, model, sizes, order, t, world)
+            except Exception as ex:  # report, do not hide
+                e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:300],
+                       "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
         del model
         R.ratel_finalize()
         torch.cuda.empty_cache()
         clocks = sampler.stop() if sampler else None
 
-        e2e = None
+        e2e_host = None
         if not args.no_e2e:
             try:
-                e2e = run_e2e(args, R, torch, dev, local, rank, world)
+                e2e_host = run_e2e(args, R, torch, dev, local, rank, world)
             except Exception as ex:  # report, do not hide
-                e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:300],
-                       "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
+                e2e_host = {"value": None, "unit": UNIT, "error": repr(ex)[:300],
+                            "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
             torch.cuda.empty_cache()
+        if e2e is None:
+            e2e = e2e_host
 
         cpu = None
         if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -712,6 +776,7 @@ def main():
                     "warmup": args.warmup, "ms_per_step": ms / args.steps, "higher_is_better": True,
                     "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
                     "config": cfgd, "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
+                    "e2e_host_states": e2e_host,
                     "clocks": dict(clocks or {}, remeasured=remeasured), "gpu_launches": launches,
                     "overlap": overlap,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
