@@ -571,3 +571,50 @@ def test_checkpoint_resume_bitwise(cuda_dev):
                 R.ratel_offload_grad_chunk(bl.id, None)
             R.ratel_sync(None)
     assert_bitwise(snapshot(a), snapshot(c))
+
+
+def test_randomized_protocol_no_side_effects(cuda_dev):
+    """Randomised call sequences: arming before/after/between hand-offs,
+    random hand-off order, and injected out-of-protocol calls (double
+    hand-off, early sync, non-increasing step, unknown block, bad
+    hyperparameters) that must fail with RATEL_ESTATE/EINVAL and change
+    nothing.  The final states equal a canonical run bit for bit."""
+    rng = np.random.default_rng(2024)
+    sizes = [[40_001], [8_192, 5], [100_000], [17]]
+    canon = _fresh(sizes, cuda_dev)
+    run(canon, 6, check_every=False)
+    blocks = _fresh(sizes, cuda_dev)
+    with ratel_lib():
+        for b in blocks:
+            b.register()
+        for t in range(1, 7):
+            for b in blocks:
+                b.load_grads(t)
+            torch.cuda.synchronize()
+            ids = list(rng.permutation([b.id for b in blocks]))
+            arm_at = int(rng.integers(0, len(ids) + 1))     # arm after this many hand-offs
+            handed = []
+            for j in range(len(ids) + 1):
+                if j == arm_at:
+                    R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+                if rng.random() < 0.5:   # inject an invalid call
+                    kind = int(rng.integers(0, 5))
+                    with pytest.raises(R.RatelError) as e:
+                        if kind == 0 and handed:
+                            R.ratel_offload_grad_chunk(int(handed[0]), None)
+                        elif kind == 1 and j < len(ids):
+                            R.ratel_sync(None)          # missing hand-offs
+                        elif kind == 1:
+                            R.ratel_offload_grad_chunk(-1, None)
+                        elif kind == 2:
+                            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t - 1 if t > 1 else 0)
+                        elif kind == 3:
+                            R.ratel_offload_grad_chunk(999, None)
+                        else:
+                            R.ratel_adam_step(-1.0, 0.9, 0.999, 1e-8, 1e-2, t + 100)
+                    assert e.value.code in (R.RATEL_ESTATE, R.RATEL_EINVAL)
+                if j < len(ids):
+                    R.ratel_offload_grad_chunk(int(ids[j]), None)
+                    handed.append(ids[j])
+            R.ratel_sync(None)
+    assert_bitwise(snapshot(canon), snapshot(blocks))
