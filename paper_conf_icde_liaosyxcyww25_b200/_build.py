@@ -55,7 +55,7 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, de
     if out is None and not force and not stale():
         return LIB
     tmp = target + f".tmp{os.getpid()}"
-    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O2,-fopenmp",
+    cmd = [_nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3,-fopenmp,-fno-math-errno",
            *[f"-D{d}" for d in defines],
            "-Xptxas", "-v" if verbose else "-O3", "-shared", "-o", tmp,
            "-I", INCLUDE, "-I", CSRC, "-I", _nccl_include(),
