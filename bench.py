@@ -386,13 +386,18 @@ def overlap_probe(args, R, torch, dev, model, sizes, order, t0):
     return res, t[0]
 
 
+HOST_ENQUEUE_MS = []   # host time to issue one step (arm + hand-offs + stream sync): never blocks
+
+
 def timed_steps(R, torch, order, stream, t0, K, pre_step=None, post_step=None):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
     for k in range(K):
         if pre_step:
             pre_step(k)
+        h0 = time.perf_counter()
         step_once(R, t0 + k, order, stream)
+        HOST_ENQUEUE_MS.append(1e3 * (time.perf_counter() - h0))
         if post_step:
             post_step(k)
     ev1.record(stream)
@@ -778,6 +783,8 @@ def main():
                     "config": cfgd, "roofline": roof, "cpu_baseline": cpu, "e2e": e2e,
                     "e2e_host_states": e2e_host,
                     "clocks": dict(clocks or {}, remeasured=remeasured), "gpu_launches": launches,
+                    "host_enqueue_ms_per_step": sorted(HOST_ENQUEUE_MS)[len(HOST_ENQUEUE_MS) // 2]
+                    if HOST_ENQUEUE_MS else None,
                     "overlap": overlap,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
             print(json.dumps(line), flush=True)
