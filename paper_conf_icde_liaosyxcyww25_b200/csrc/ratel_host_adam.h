@@ -3,8 +3,9 @@
 // PAPER.md §IV-C: "the CPU updates the model states of the tensor i and
 // produces a 16-bit parameter copy", on a CPU optimizer that
 // keeps P32/OS32 in main memory.  This is that
-// handler for one rank slice of one range: double-precision arithmetic on the
-// fp32 states in pinned host memory, bf16 RNE of the stored fp32 master.
+// handler for one rank slice of one range: fp32 arithmetic (double for the
+// Adam-L2 gradient) on the fp32 states in pinned host memory, bf16 RNE of the
+// stored fp32 master.
 #pragma once
 
 #include <stddef.h>
