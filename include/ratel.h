@@ -85,7 +85,7 @@ enum {
  *   HOST_COMPUTE  the paper's own design (§IV-C; CPU optimizer
  *                 P:L582-584): states in page-locked host memory, G16 copied
  *                 device->host (2 B/param), the CPU updates the states and
- *                 produces P16 (double arithmetic, OpenMP), P16 copied
+ *                 produces P16 (fp32 arithmetic, SIMD + OpenMP), P16 copied
  *                 host->device (2 B/param); stream-ordered via
  *                 cudaLaunchHostFunc, the host thread never blocks. */
 typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2 } ratel_residency;

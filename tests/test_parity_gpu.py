@@ -453,7 +453,7 @@ def test_clip_adam_l2_pinned_host(cuda_dev):
 # ------------------------------------------- HOST_COMPUTE (the paper's CPU handler)
 @pytest.mark.parametrize("mode,max_norm", [(oracle.ADAMW, 0.0), (oracle.ADAM_L2, 0.0), (oracle.ADAMW, 1e-3)])
 def test_host_compute_vs_oracle(cuda_dev, mode, max_norm):
-    """RATEL_HOST_COMPUTE: G16 D2H, CPU AdamW in double on the pinned states,
+    """RATEL_HOST_COMPUTE: G16 D2H, CPU AdamW (fp32, SIMD) on the pinned states,
     P16 H2D (§IV-C) -- ragged multi-range blocks, 5 steps."""
     blocks = [GpuBlock(0, [789_760 + 3, 256], cuda_dev, host_compute=True, wd_flags=[1, 0]),
               GpuBlock(1, [65_537], cuda_dev, host_compute=True)]
