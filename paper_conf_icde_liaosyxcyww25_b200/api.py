@@ -81,7 +81,10 @@ class _Range:
 
 
 class Ratel_Optimizer:
-    """AdamW (or Adam-L2) over flat per-block buffers, driven by hand-offs."""
+    """AdamW (or Adam-L2) over flat per-block buffers, driven by hand-offs.
+
+    residency: "device" (states in HBM), "host" (pinned host, GPU-streamed) or
+    "hostcompute" (pinned host, the paper's CPU handler)."""
 
     def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,
                  residency="device", no_decay=None, first_block_id=0):
@@ -103,7 +106,8 @@ class Ratel_Optimizer:
             ranges = [_Range(ps, wd, world, rank, dev, residency) for ps, wd in groups if ps]
             bid = first_block_id + j
             R.ratel_register_block(bid, [r.ratel_range() for r in ranges],
-                                   R.RATEL_DEVICE if residency == "device" else R.RATEL_PINNED_HOST)
+                                   {"device": R.RATEL_DEVICE, "host": R.RATEL_PINNED_HOST,
+                                    "hostcompute": R.RATEL_HOST_COMPUTE}[residency])
             self.blocks.append(ranges)
             self.block_ids.append(bid)
         self._pending = {}
@@ -153,6 +157,33 @@ class Ratel_Optimizer:
                 self._handed.add(bid)
                 R.ratel_offload_grad_chunk(bid, s)
         R.ratel_sync(s)
+
+    def state_dict(self) -> dict:
+        """Step counter and copies of every range's fp32 master/exp_avg/
+        exp_avg_sq (this rank's slices).  Call between steps."""
+        torch.cuda.synchronize()
+        return {"t": self.t, "lr": self.lr, "betas": self.betas, "eps": self.eps,
+                "weight_decay": self.weight_decay,
+                "ranges": [[{"master": r.master.detach().cpu().clone(), "exp_avg": r.m.detach().cpu().clone(),
+                             "exp_avg_sq": r.v.detach().cpu().clone()} for r in ranges] for ranges in self.blocks]}
+
+    def load_state_dict(self, sd: dict) -> None:
+        """Restore states saved by state_dict() (same block/range layout) and
+        refresh P16 = bf16(master) through the library on the next step; the
+        step counter continues from sd["t"].  Call between steps."""
+        assert len(sd["ranges"]) == len(self.blocks)
+        for ranges, saved in zip(self.blocks, sd["ranges"]):
+            assert len(ranges) == len(saved)
+            for r, s in zip(ranges, saved):
+                r.master.copy_(s["master"])
+                r.m.copy_(s["exp_avg"])
+                r.v.copy_(s["exp_avg_sq"])
+                beg, end = r.slice
+                if end > beg:  # the model's working copy must match the restored master
+                    r.p16[beg:end].copy_(r.master[:end - beg].to(r.p16.device).to(torch.bfloat16))
+        self.t = int(sd["t"])
+        self.lr, self.betas, self.eps, self.weight_decay = sd["lr"], tuple(sd["betas"]), sd["eps"], sd["weight_decay"]
+        torch.cuda.synchronize()
 
     def state(self, block_index: int):
         """(master, exp_avg, exp_avg_sq, p16, g16) flat views of each range of a block."""

@@ -64,3 +64,46 @@ def test_paper_api_matches_oracle(cuda_dev):
         assert R.ratel_launch_count() - launches0 == 4 * nb
         opt.remove_hooks()
         del opt
+
+
+def test_paper_api_state_dict_resume(cuda_dev):
+    """Ratel_Optimizer.state_dict()/load_state_dict(): 3 steps, save, rebuild
+    model + optimizer from the saved states, 2 more steps == 5 straight steps."""
+    def build():
+        torch.manual_seed(1)
+        return torch.nn.Sequential(*[Block(64) for _ in range(2)]).to(cuda_dev)
+
+    x = torch.randn(32, 64, device=cuda_dev, dtype=torch.bfloat16)
+
+    def train(model, opt, n):
+        for _ in range(n):
+            opt.begin_step()
+            model(x).float().pow(2).mean().backward()
+            opt.end_step()
+        torch.cuda.synchronize()
+
+    def snap(opt):
+        return [t.cpu().clone() for ranges in opt.blocks for r in ranges for t in (r.master, r.m, r.v, r.p16)]
+
+    with Ratel_init():
+        m1 = build()
+        o1 = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in m1]))
+        train(m1, o1, 5)
+        want = snap(o1)
+        o1.remove_hooks()
+    with Ratel_init():
+        m2 = build()
+        o2 = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in m2]))
+        train(m2, o2, 3)
+        sd = o2.state_dict()
+        o2.remove_hooks()
+    with Ratel_init():
+        m3 = build()
+        o3 = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in m3]))
+        o3.load_state_dict(sd)
+        train(m3, o3, 2)
+        got = snap(o3)
+        o3.remove_hooks()
+    for a, b in zip(want, got):
+        assert torch.equal(a.view(torch.int16) if a.dtype == torch.bfloat16 else a.view(torch.int32),
+                           b.view(torch.int16) if b.dtype == torch.bfloat16 else b.view(torch.int32))
