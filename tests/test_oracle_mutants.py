@@ -1,0 +1,148 @@
+"""Mutation check of the oracle's pins (CPU).
+
+Each mutant is ratel_oracle.c with ONE plausible mistake (a dropped term, a
+wrong sign, a wrong index/power, a transposed operand, the other eps reading,
+truncating instead of rounding), compiled to a temp dir.  The pins of
+tests/test_oracle_pins.py are re-run against it in a compact form: every
+mutant must be caught by at least one pin, otherwise the pins would not be
+pinning that part of the oracle.
+"""
+import ctypes
+import math
+import os
+import subprocess
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+
+SRC = os.path.join(os.path.dirname(oracle.__file__), "ratel_oracle.c")
+
+MUTANTS = {
+    "eps_inside_sqrt": ("(sqrt(vv / bc2) + hp->eps)", "sqrt(vv / bc2 + hp->eps)"),
+    "kingma_efficient_eps": ("(sqrt(vv / bc2) + hp->eps)", "(sqrt(vv / bc2) + hp->eps / sqrt(1.0 - hp->beta2))"),
+    "bias1_uses_t_minus_1": ("double bc1 = 1.0 - pow(hp->beta1, t);", "double bc1 = 1.0 - pow(hp->beta1, t - 1.0 + 1e-300);"),
+    "no_bias2": ("double bc2 = 1.0 - pow(hp->beta2, t);", "double bc2 = 1.0;"),
+    "beta2_swapped": ("double vv = hp->beta2 * (*v) + (1.0 - hp->beta2) * g * g;",
+                      "double vv = (1.0 - hp->beta2) * (*v) + hp->beta2 * g * g;"),
+    "m_drops_1_minus_beta1": ("(1.0 - hp->beta1) * g;", "g;"),
+    "wd_sign": ("th = th * (1.0 - hp->lr * hp->weight_decay);", "th = th * (1.0 + hp->lr * hp->weight_decay);"),
+    "wd_without_lr": ("th = th * (1.0 - hp->lr * hp->weight_decay);", "th = th * (1.0 - hp->weight_decay);"),
+    "l2_sign": ("g = g + hp->weight_decay * th;", "g = g - hp->weight_decay * th;"),
+    "update_sign": ("th = th - delta;", "th = th + delta;"),
+    "bf16_truncates": ("if (rem > 0x8000u) return (uint16_t)(lo + 1);", "if (rem > 0xFFFFu) return (uint16_t)(lo + 1);"),
+    "bf16_ties_away": ("return (lo & 1u) ? (uint16_t)(lo + 1) : lo;", "return (uint16_t)(lo + 1);"),
+    "p16_from_wrong_array": ("p16[i] = oracle_bf16_rne(p32[i]);", "p16[i] = oracle_bf16_rne(m32[i]);"),
+    "clip_not_clamped": ("return (c < 1.0 || isnan(c)) ? c : 1.0;", "return c;"),
+    "clip_norm_squared": ("double c = max_norm / (sqrt(sumsq) + 1e-6);", "double c = max_norm / (sumsq + 1e-6);"),
+    "sumsq_abs": ("s += g * g;", "s += fabs(g);"),
+}
+
+
+def _build_mutant(tmp_path, name, old, new):
+    src = open(SRC).read()
+    assert src.count(old) == 1, (name, old)
+    path = tmp_path / f"{name}.c"
+    path.write_text(src.replace(old, new))
+    so = tmp_path / f"lib{name}.so"
+    subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared", "-std=c11",
+                           "-o", str(so), str(path), "-lm"])
+    return str(so)
+
+
+def _with_lib(path):
+    """Point the oracle wrapper at another build for the duration of a check."""
+    saved = oracle._lib
+    oracle._lib = None
+    real_build = oracle.build
+    oracle.build = lambda force=False: path
+    try:
+        oracle.lib()
+    finally:
+        oracle.build = real_build
+    return saved
+
+
+def _pins_pass():
+    """Compact versions of the oracle pins; True iff all hold."""
+    f32ulp = lambda x: np.spacing(np.abs(np.float32(x))).astype(np.float64)
+    lr, eps = 1e-3, 1e-8
+    try:
+        # step-1 closed form, AdamW with decay, and the eps separator
+        n = 2048
+        th0 = synth.theta0(n, block=3)
+        g = synth.grad16(n, step=1, block=3)
+        for wd in (0.0, 1e-2):
+            r = oracle.Range.fresh(th0)
+            oracle.adam_range(r, g, oracle.hparams(step=1, weight_decay=wd))
+            gd = synth.bf16_bits_to_f32(g).astype(np.float64)
+            exp = th0.astype(np.float64) * (1 - lr * wd) - lr * gd / (np.abs(gd) + eps)
+            if not np.all(np.abs(r.p32 - exp) <= f32ulp(exp)):
+                return False
+        # Adam-L2 step 1
+        r = oracle.Range.fresh(th0)
+        oracle.adam_range(r, g, oracle.hparams(step=1, mode=oracle.ADAM_L2))
+        gp = synth.bf16_bits_to_f32(g).astype(np.float64) + 1e-2 * th0.astype(np.float64)
+        exp = th0.astype(np.float64) - lr * gp / (np.abs(gp) + eps)
+        if not np.all(np.abs(r.p32 - exp) <= f32ulp(exp)):
+            return False
+        # constant gradient over 10 steps (bias corrections at every t)
+        vals = np.array([2.0 ** -10, -(2.0 ** -20), 3 * 2.0 ** -15, -(2.0 ** -8)], np.float32)
+        cb = (vals.view(np.uint32) >> 16).astype(np.uint16)
+        r = oracle.Range.fresh(np.array([0.01, -0.02, 0.03, 0.0], np.float32))
+        for t in range(1, 11):
+            oracle.adam_range(r, cb, oracle.hparams(step=t, weight_decay=0.0))
+        exp = np.array([0.01, -0.02, 0.03, 0.0]) - 10 * lr * vals / (np.abs(vals.astype(np.float64)) + eps)
+        if not np.all(np.abs(r.p32 - exp) <= 10 * f32ulp(np.abs(exp) + 10 * lr)):
+            return False
+        # torch.optim.AdamW, 10 steps, fp32 storage emulated (R13 bound 1e-6)
+        from tests.tolerance import check_range
+        from tests.test_oracle_pins import _torch_run
+        n, T = 20_000, 6
+        th0 = synth.theta0(n, block=11)
+        grads = [synth.grad16(n, step=t, block=11) for t in range(1, T + 1)]
+        r = oracle.Range.fresh(th0)
+        for t, gg in enumerate(grads, start=1):
+            oracle.adam_range(r, gg, oracle.hparams(step=t))
+        tp, tm, tv, _ = _torch_run(th0, grads, oracle.ADAMW)
+        check_range(dict(p32=tp, m32=tm, v32=tv, p16=oracle.bf16_rne(tp)), r, tol=1e-6)
+        # clip vs torch clip_grad_norm_
+        S = oracle.grad_sumsq(grads[0])
+        tn = float(torch.linalg.vector_norm(torch.from_numpy(synth.bf16_bits_to_f32(grads[0]).astype(np.float64))))
+        if abs(math.sqrt(S) - tn) > 1e-12 * tn:
+            return False
+        if oracle.clip_coef(1e-12, 1.0) != 1.0 or abs(oracle.clip_coef(4.0, 1.0) - 1 / (2 + 1e-6)) > 1e-15:
+            return False
+        # bf16 rounding against torch's cast on random patterns + all ties
+        u = np.random.default_rng(0).integers(0, 2 ** 32, 1 << 18, dtype=np.uint64).astype(np.uint32)
+        ties = ((np.arange(1 << 16, dtype=np.uint32) << 16) | 0x8000).astype(np.uint32)
+        x = np.concatenate([u, ties]).view(np.float32)
+        x = x[np.isfinite(x)]
+        mine = oracle.bf16_rne(x)
+        ref = torch.from_numpy(x).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+        if not np.array_equal(mine, ref):
+            return False
+        # no staleness: P16 == bf16_rne(stored P32)
+        if not np.array_equal(r.p16, oracle.bf16_rne(r.p32)):
+            return False
+    except AssertionError:
+        return False
+    return True
+
+
+def test_unmutated_oracle_passes_the_compact_pins():
+    assert _pins_pass()
+
+
+@pytest.mark.parametrize("name", sorted(MUTANTS))
+def test_every_mutant_is_caught(tmp_path, name):
+    old, new = MUTANTS[name]
+    so = _build_mutant(tmp_path, name, old, new)
+    saved = _with_lib(so)
+    try:
+        assert not _pins_pass(), f"mutant {name} survived the pins"
+    finally:
+        oracle._lib = saved
