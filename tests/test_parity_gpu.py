@@ -618,3 +618,53 @@ def test_randomized_protocol_no_side_effects(cuda_dev):
                     handed.append(ids[j])
             R.ratel_sync(None)
     assert_bitwise(snapshot(canon), snapshot(blocks))
+
+
+def test_fullsize_13b_model_sampled_vs_oracle(cuda_dev):
+    """The whole BASELINE configs[1] model (13B GPT states: 40 x 314,639,360 +
+    262,568,960 params, 180 GB resident) in bench.py's launch configuration
+    (one flat range per block, AGO order, 2-slot gradient ring recycled with
+    ratel_block_wait), 3 steps with device-generated inputs; 4096 sampled
+    elements per block vs the oracle computed one by one, plus the first and
+    last 8 elements of every block (tails)."""
+    import bench
+    sizes = bench.model_blocks("13B")
+    assert sum(sizes) == 12_848_143_360
+    steps = 3
+    rng = np.random.default_rng(11)
+    samples = [np.unique(np.concatenate([np.arange(8), np.arange(n - 8, n),
+                                         rng.integers(0, n, 4096)])).astype(np.uint64) for n in sizes]
+    refs = [oracle.Range.fresh(synth.theta0_at(idx, block=b)) for b, idx in enumerate(samples)]
+    cap = max(sizes)
+    ring = [torch.empty(cap, dtype=torch.bfloat16, device=cuda_dev) for _ in range(2)]
+    states = []
+    with ratel_lib():
+        for b, n in enumerate(sizes):
+            th = torch.empty(n, dtype=torch.float32, device=cuda_dev)
+            R.ratel_gen_theta0(th.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, b))
+            m = torch.zeros(n, device=cuda_dev)
+            v = torch.zeros(n, device=cuda_dev)
+            p = torch.zeros(n, dtype=torch.bfloat16, device=cuda_dev)
+            states.append((p, th, m, v))
+            R.ratel_register_block(b, [R.make_range(p, ring[b % 2], th, m, v, n)], R.RATEL_DEVICE)
+        s = torch.cuda.Stream()
+        order = list(reversed(range(len(sizes))))
+        for t in range(1, steps + 1):
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            for j, b in enumerate(order):
+                if j >= 2:
+                    R.ratel_block_wait(order[j - 2], s)              # ring slot consumed
+                R.ratel_gen_grad16(ring[b % 2].data_ptr(), sizes[b], 0,
+                                   R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, b), s)
+                R.ratel_offload_grad_chunk(b, s)
+            R.ratel_sync(None)
+            for b, idx in enumerate(samples):
+                oracle.adam_range(refs[b], synth.grad16_at(idx, step=t, block=b), oracle.hparams(step=t))
+        for b, idx in enumerate(samples):
+            p, th, m, v = states[b]
+            ii = torch.from_numpy(idx.astype(np.int64)).to(cuda_dev)
+            got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
+                       p16=torch_to_u16(p[ii]))
+            check_range(got, refs[b], own_rne=oracle.bf16_rne, what=f"13B block {b}")
+            assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
+        del states
