@@ -211,6 +211,33 @@ def workload_config(args, world):
             "max_grad_norm": args.clip}
 
 
+class PinnedArena:
+    """One exact-size page-locked host buffer from ratel_alloc_pinned
+    (cudaHostAlloc): torch's pinned allocator rounds large blocks up, which
+    would not fit 100+ GB of host states into the box's RAM."""
+
+    def __init__(self, torch, nfloats):
+        import paper_conf_icde_liaosyxcyww25_b200 as R
+        self.torch = torch
+        self.owner = R.pinned_tensor(max(nfloats, 8))
+        self.t = self.owner.tensor
+        self.t.zero_()
+        self.off = 0
+
+    def take(self, n):
+        v = self.t[self.off:self.off + n]
+        self.off += (n + 7) // 8 * 8          # keep every slice 32-byte aligned
+        return v
+
+    def close(self):
+        if self.t is not None:
+            self.torch.cuda.synchronize()
+            self.t = None
+            self.owner = None   # ratel_free_pinned
+
+    __del__ = close
+
+
 class Model:
     """Synthetic model states of one rank: per block one flat range.
     symm=True allocates P16 in torch symmetric memory (peer-mapped) for the
@@ -228,6 +255,13 @@ class Model:
             R.ratel_gen_grad16(g.data_ptr(), cap_max, 0, key)
         self.p16 = []
         self.peer_ptrs = []
+        self.arenas = []
+        if residency != "device":
+            own_total = 0
+            for n in sizes:
+                beg, end = R.ratel_rank_slice(n, world, rank)
+                own_total += (max(end - beg, 8) + 7) // 8 * 8
+            self.arenas = [PinnedArena(torch, own_total) for _ in range(3)]
         for b, n in enumerate(sizes):
             cap = R.ratel_padded_numel(n, world)
             beg, end = R.ratel_rank_slice(n, world, rank)
@@ -249,11 +283,9 @@ class Model:
             else:
                 tmp = torch.empty(s, dtype=torch.float32, device=dev)
                 R.ratel_gen_theta0(tmp.data_ptr(), end - beg, beg, R.ratel_gen_stream_key(0x5EED5EED, 1, 0, b))
-                th = torch.empty(s, dtype=torch.float32, pin_memory=True)
+                th, m, v = (a.take(s) for a in self.arenas)
                 th.copy_(tmp)
                 del tmp
-                m = torch.zeros(s, dtype=torch.float32, pin_memory=True)
-                v = torch.zeros(s, dtype=torch.float32, pin_memory=True)
             g = self.grad_ring[b % grad_ring]
             self.ranges.append(R.make_range(p, g, th, m, v, n))
             self.keep.append((p, th, m, v))

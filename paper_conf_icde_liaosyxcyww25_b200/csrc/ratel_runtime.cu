@@ -982,4 +982,28 @@ int ratel_kernel_timing(double* total_ms, int64_t* launches, int reset) {
 
 int64_t ratel_launch_count(void) { return G.launches; }
 
+int ratel_alloc_pinned(uint64_t bytes, void** out) {
+  if (out == nullptr) return set_error(RATEL_EINVAL, "ratel_alloc_pinned: NULL");
+  *out = nullptr;
+  if (bytes == 0) return set_error(RATEL_EINVAL, "ratel_alloc_pinned: 0 bytes");
+  const cudaError_t e = cudaHostAlloc(out, bytes, cudaHostAllocPortable);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    *out = nullptr;
+    return set_error(RATEL_ENOMEM, "cudaHostAlloc(%llu) failed: %s", static_cast<unsigned long long>(bytes),
+                     cudaGetErrorString(e));
+  }
+  return RATEL_OK;
+}
+
+int ratel_free_pinned(void* p) {
+  if (p == nullptr) return RATEL_OK;
+  const cudaError_t e = cudaFreeHost(p);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_error(RATEL_EINVAL, "cudaFreeHost failed: %s", cudaGetErrorString(e));
+  }
+  return RATEL_OK;
+}
+
 }  // extern "C"

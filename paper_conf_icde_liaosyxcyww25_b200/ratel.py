@@ -100,6 +100,8 @@ def load_library(path: str = _LIB_PATH, strict: bool = True):
         "ratel_get_grad_sumsq": (I, [ctypes.POINTER(D)]),
         "ratel_kernel_timing": (I, [ctypes.POINTER(D), ctypes.POINTER(ctypes.c_int64), I]),
         "ratel_launch_count": (ctypes.c_int64, []),
+        "ratel_alloc_pinned": (I, [U64, ctypes.POINTER(P)]),
+        "ratel_free_pinned": (I, [P]),
         "ratel_gen_stream_key": (U64, [U64, U64, U64, U64]),
         "ratel_gen_theta0": (I, [P, U64, U64, U64, P]),
         "ratel_gen_grad16": (I, [P, U64, U64, U64, P]),
@@ -224,6 +226,35 @@ def ratel_kernel_timing(reset: bool = False) -> tuple[float, int]:
 
 def ratel_launch_count() -> int:
     return int(_lib.ratel_launch_count())
+
+
+def ratel_alloc_pinned(nbytes: int) -> int:
+    out = ctypes.c_void_p()
+    _check(_lib.ratel_alloc_pinned(nbytes, ctypes.byref(out)))
+    return int(out.value)
+
+
+def ratel_free_pinned(ptr: int) -> None:
+    _check(_lib.ratel_free_pinned(ptr))
+
+
+def pinned_tensor(nfloats: int):
+    """An fp32 CPU tensor over exact-size page-locked memory from
+    ratel_alloc_pinned (freed when the returned owner is collected)."""
+    import numpy as np
+    import torch
+
+    class _Owner:
+        def __init__(self, n):
+            self.ptr = ratel_alloc_pinned(n * 4)
+            buf = (ctypes.c_float * n).from_address(self.ptr)
+            self.tensor = torch.from_numpy(np.ctypeslib.as_array(buf))
+
+        def __del__(self):
+            if getattr(self, "ptr", 0):
+                ratel_free_pinned(self.ptr)
+                self.ptr = 0
+    return _Owner(nfloats)
 
 
 # -------------------------------------------------- include/ratel_gen.h

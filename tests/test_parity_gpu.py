@@ -668,3 +668,33 @@ def test_fullsize_13b_model_sampled_vs_oracle(cuda_dev):
             check_range(got, refs[b], own_rne=oracle.bf16_rne, what=f"13B block {b}")
             assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
         del states
+
+
+def test_alloc_pinned_states(cuda_dev):
+    """ratel_alloc_pinned: exact-size page-locked host memory accepted as
+    RATEL_PINNED_HOST / RATEL_HOST_COMPUTE states; results equal the device
+    residency bit for bit."""
+    n = 300_001
+    ref = _fresh([[n]], cuda_dev)
+    run(ref, 2, check_every=False)
+    for residency in (R.RATEL_PINNED_HOST, R.RATEL_HOST_COMPUTE):
+        b = GpuBlock(0, [n], cuda_dev)
+        owners = [R.pinned_tensor(n) for _ in range(3)]
+        for o, src in zip(owners, (b.master[0], b.m[0], b.v[0])):
+            o.tensor.copy_(src.cpu())
+        b.master[0], b.m[0], b.v[0] = (o.tensor for o in owners)
+        with ratel_lib():
+            R.ratel_register_block(0, b.ranges(), residency)
+            for t in (1, 2):
+                b.load_grads(t)
+                torch.cuda.synchronize()
+                R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+                R.ratel_offload_grad_chunk(0, None)
+                R.ratel_sync(None)
+        got, want = b.gpu_state(0), ref[0].gpu_state(0)
+        if residency == R.RATEL_PINNED_HOST:   # same kernel: bitwise
+            assert np.array_equal(got["p32"].view(np.uint32), want["p32"].view(np.uint32))
+            assert np.array_equal(got["p16"], want["p16"])
+        else:                                   # CPU handler: within the R13 bounds
+            check_range(got, ref[0].oracle[0], own_rne=oracle.bf16_rne)
+        del owners
