@@ -362,8 +362,15 @@ __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t b
 }
 
 __device__ __forceinline__ void bulk_store(void* dst, const void* src, uint32_t bytes) {
+#if RATEL_TMA_EVICT_FIRST
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;"
+               ::"l"(dst), "r"(smem_u32(src)), "r"(bytes), "l"(pol) : "memory");
+#else
   asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;"
                ::"l"(dst), "r"(smem_u32(src)), "r"(bytes) : "memory");
+#endif
 }
 
 // Tile k of the concatenation of the ranges' vector bodies (n & ~7 each).
