@@ -69,6 +69,11 @@ def lib():
         _lib.oracle_grad_sumsq.restype = ctypes.c_double
         _lib.oracle_clip_coef.argtypes = [ctypes.c_double, ctypes.c_double]
         _lib.oracle_clip_coef.restype = ctypes.c_double
+        _lib.oracle_reduce_grads.argtypes = [ctypes.c_size_t, P, ctypes.c_int, ctypes.c_double, P]
+        _lib.oracle_adam_range_gd.argtypes = [ctypes.c_size_t, P, ctypes.c_double, ctypes.c_int,
+                                              ctypes.POINTER(HParams), P, P, P, P, P, P]
+        _lib.oracle_grad_sumsq_d.argtypes = [P, ctypes.c_size_t, ctypes.c_double]
+        _lib.oracle_grad_sumsq_d.restype = ctypes.c_double
     return _lib
 
 
@@ -153,6 +158,49 @@ def adam_step(ranges, grads, hp: HParams, max_grad_norm: float = 0.0, threads: i
         coef = clip_coef(S, max_grad_norm)
     for r, g in zip(ranges, grads):
         adam_range(r, g, hp, coef, threads)
+    return S, coef
+
+
+def reduce_grads(g16s, scale: float) -> np.ndarray:
+    """Data-parallel gradient of a range: scale * sum over ranks (R17), double."""
+    gs = [np.ascontiguousarray(g, dtype=np.uint16) for g in g16s]
+    n = gs[0].size
+    for g in gs:
+        _check(g, np.uint16, n)
+    ptrs = (ctypes.c_void_p * len(gs))(*[g.ctypes.data for g in gs])
+    out = np.empty(n, np.float64)
+    lib().oracle_reduce_grads(n, ptrs, len(gs), scale, _ptr(out))
+    return out
+
+
+def adam_range_gd(r: Range, gd: np.ndarray, hp: HParams, coef: float = 1.0) -> None:
+    """In-place update of one range from a double gradient (fp32 storage)."""
+    n = r.p32.size
+    gd = np.ascontiguousarray(gd, dtype=np.float64)
+    _check(gd, np.float64, n)
+    lib().oracle_adam_range_gd(n, _ptr(gd), coef, r.apply_wd, ctypes.byref(hp), _ptr(r.p32),
+                               _ptr(r.m32), _ptr(r.v32), _ptr(r.p16), _ptr(r.theta_bar), _ptr(r.m_bar))
+
+
+def grad_sumsq_d(gd: np.ndarray, s0: float = 0.0) -> float:
+    gd = np.ascontiguousarray(gd, dtype=np.float64)
+    return lib().oracle_grad_sumsq_d(_ptr(gd), gd.size, s0)
+
+
+def adam_step_dp(ranges, rank_grads, scale: float, hp: HParams, max_grad_norm: float = 0.0):
+    """One synchronous step with the data-parallel gradient reduction (R17):
+    rank_grads[k] is the list of every rank's bf16 grad of range k.  Returns
+    (sumsq, coef) like adam_step."""
+    gds = [reduce_grads(gq, scale) for gq in rank_grads]
+    S = None
+    coef = 1.0
+    if max_grad_norm > 0:
+        S = 0.0
+        for gd in gds:
+            S = grad_sumsq_d(gd, S)
+        coef = clip_coef(S, max_grad_norm)
+    for r, gd in zip(ranges, gds):
+        adam_range_gd(r, gd, hp, coef)
     return S, coef
 
 

@@ -162,3 +162,42 @@ double oracle_clip_coef(double sumsq, double max_norm) {
   double c = max_norm / (sqrt(sumsq) + 1e-6);
   return (c < 1.0 || isnan(c)) ? c : 1.0; /* NaN propagates like torch.clamp */
 }
+
+/* ---- Data-parallel gradient reduction (R17) ----
+ * With the reduce-scatter fused into the update, the gradient of element i is
+ * the data-parallel combination of the N ranks' local bf16 gradients,
+ *     g[i] = scale * sum_{q=0..nq-1} (double) bf16(G16_q[i]),
+ * summed in double in rank order (scale = 1/N gives DDP's mean, 1 the sum).
+ * The paper leaves multi-GPU gradient semantics unspecified;
+ * this is the plain definition of a sum/mean all-reduce, written out. */
+void oracle_reduce_grads(size_t n, const uint16_t* const* g16s, int nq, double scale, double* out) {
+  for (size_t i = 0; i < n; ++i) {
+    double s = 0.0;
+    for (int q = 0; q < nq; ++q) s = s + oracle_bf16_to_double(g16s[q][i]);
+    out[i] = scale * s;
+  }
+}
+
+/* The update of oracle_adam_range from a double gradient (the reduced one):
+ * the same per-element steps, g = g[i] * coef instead of the widened bf16. */
+void oracle_adam_range_gd(size_t n, const double* gd, double coef, int apply_wd,
+                          const oracle_hparams* hp, float* p32, float* m32, float* v32,
+                          uint16_t* p16, double* theta_bar, double* m_bar) {
+  for (size_t i = 0; i < n; ++i) {
+    double g = gd[i] * coef;
+    double th = (double)p32[i], m = (double)m32[i], v = (double)v32[i], gu;
+    double ad = adam_elem(g, &th, &m, &v, apply_wd, hp, &gu);
+    p32[i] = (float)th;
+    m32[i] = (float)m;
+    v32[i] = (float)v;
+    p16[i] = oracle_bf16_rne(p32[i]);
+    update_scales(i, gu, ad, apply_wd, hp, theta_bar, m_bar);
+  }
+}
+
+/* Sum of squares of a double gradient, in index order, continuing s0. */
+double oracle_grad_sumsq_d(const double* g, size_t n, double s0) {
+  double s = s0;
+  for (size_t i = 0; i < n; ++i) s += g[i] * g[i];
+  return s;
+}

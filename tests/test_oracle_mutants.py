@@ -39,12 +39,18 @@ MUTANTS = {
     "clip_not_clamped": ("return (c < 1.0 || isnan(c)) ? c : 1.0;", "return c;"),
     "clip_norm_squared": ("double c = max_norm / (sqrt(sumsq) + 1e-6);", "double c = max_norm / (sumsq + 1e-6);"),
     "sumsq_abs": ("s += g * g;", "s += fabs(g);"),
+    # data-parallel gradient reduction (R17)
+    "dp_no_scale": ("out[i] = scale * s;", "out[i] = s;"),
+    "dp_first_rank_only": ("for (int q = 0; q < nq; ++q)", "for (int q = 0; q < 1; ++q)"),
+    "dp_drops_last_rank": ("for (int q = 0; q < nq; ++q)", "for (int q = 0; q < nq - 1; ++q)"),
+    "dp_ignores_clip_coef": ("double g = gd[i] * coef;", "double g = gd[i];"),
+    "dp_sumsq_abs": ("s += g[i] * g[i];", "s += fabs(g[i]);"),
 }
 
 
 def _build_mutant(tmp_path, name, old, new):
     src = open(SRC).read()
-    assert src.count(old) == 1, (name, old)
+    assert src.count(old) >= 1, (name, old)  # every occurrence is mutated
     path = tmp_path / f"{name}.c"
     path.write_text(src.replace(old, new))
     so = tmp_path / f"lib{name}.so"
@@ -128,6 +134,33 @@ def _pins_pass():
         # no staleness: P16 == bf16_rne(stored P32)
         if not np.array_equal(r.p16, oracle.bf16_rne(r.p32)):
             return False
+        # data-parallel reduction: exact sum x scale, then torch AdamW + clip on the mean
+        N, n = 3, 4000
+        gq = [synth.grad16(n, step=1, block=31 + 100 * q) for q in range(N)]
+        vals = np.stack([synth.bf16_bits_to_f32(g).astype(np.float64) for g in gq])
+        if not np.array_equal(oracle.reduce_grads(gq, 0.5), np.array([math.fsum(vals[:, i]) for i in range(n)]) * 0.5):
+            return False
+        th0 = synth.theta0(n, block=31)
+        r = oracle.Range.fresh(th0)
+        p = torch.nn.Parameter(torch.from_numpy(th0.astype(np.float64)))
+        opt = torch.optim.AdamW([p], lr=lr, weight_decay=1e-2, foreach=False)
+        for t in (1, 2):
+            gq = [synth.grad16(n, step=t, block=31 + 100 * q) for q in range(N)]
+            S, _ = oracle.adam_step_dp([r], [gq], 1.0 / N, oracle.hparams(step=t), max_grad_norm=1e-4)
+            p.grad = sum(torch.from_numpy(synth.bf16_bits_to_f32(g).astype(np.float64)) for g in gq) / N
+            tn = float(torch.nn.utils.clip_grad_norm_([p], 1e-4, foreach=False))
+            if abs(math.sqrt(S) - tn) > n * 2.0 ** -53 * tn:
+                return False
+            opt.step()
+            with torch.no_grad():
+                p.copy_(p.float().double())
+                st = opt.state[p]
+                st["exp_avg"].copy_(st["exp_avg"].float().double())
+                st["exp_avg_sq"].copy_(st["exp_avg_sq"].float().double())
+        st = opt.state[p]
+        tp = p.detach().float().numpy()
+        check_range(dict(p32=tp, m32=st["exp_avg"].float().numpy(), v32=st["exp_avg_sq"].float().numpy(),
+                         p16=oracle.bf16_rne(tp)), r, tol=1e-6)
     except AssertionError:
         return False
     return True

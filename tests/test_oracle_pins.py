@@ -298,3 +298,77 @@ def test_oracle_regression_digests():
     spec.loader.exec_module(mg)
     want = json.load(open(os.path.join(here, "oracle_digests.json")))["sha256"]
     assert mg.digests() == want
+
+
+# ------------------------------------- data-parallel gradient reduction (R17)
+def _rank_grads(n, N, step=1, block=21):
+    return [synth.grad16(n, step=step, block=block + 100 * q) for q in range(N)]
+
+
+@pytest.mark.parametrize("N,scale", [(2, 0.5), (4, 0.25), (3, 1.0 / 3.0), (8, 1.0)])
+def test_dp_reduce_is_the_exact_sum(N, scale):
+    """scale * sum_q g_q: for these inputs (exponents within 24 binades) the
+    double sum is exact, so it must equal math.fsum (the correctly rounded
+    sum) times scale, element by element."""
+    n = 3000
+    gq = _rank_grads(n, N)
+    got = oracle.reduce_grads(gq, scale)
+    vals = np.stack([synth.bf16_bits_to_f32(g).astype(np.float64) for g in gq])
+    exp = np.array([math.fsum(vals[:, i]) for i in range(n)]) * scale
+    assert np.array_equal(got, exp)
+
+
+@pytest.mark.parametrize("N", [1, 2, 4, 8])
+def test_dp_identical_replicas_reduce_to_the_plain_step(N):
+    """N identical replicas averaged (scale 1/N, exact) give exactly the
+    single-gradient update -- the special case that is the pinned step."""
+    n, T = 5000, 3
+    th0 = synth.theta0(n, block=22)
+    a = oracle.Range.fresh(th0)
+    b = oracle.Range.fresh(th0)
+    for t in range(1, T + 1):
+        g = synth.grad16(n, step=t, block=22)
+        hp = oracle.hparams(step=t)
+        oracle.adam_range(a, g, hp)
+        oracle.adam_range_gd(b, oracle.reduce_grads([g] * N, 1.0 / N), hp)
+    for k in ("p32", "m32", "v32", "p16", "theta_bar", "m_bar"):
+        assert np.array_equal(getattr(a, k), getattr(b, k)), k
+
+
+@pytest.mark.parametrize("clip", [0.0, 1e-3])
+def test_dp_vs_torch_mean_of_replica_grads(clip):
+    """torch.optim.AdamW (float64, fp32 storage emulated) on p.grad = the
+    mean of N ranks' grads (what DDP hands the optimizer), optionally
+    clip_grad_norm_ on that mean: R13 bound 1e-6."""
+    n, T, N = 20_000, 5, 4
+    th0 = synth.theta0(n, block=23)
+    steps = [_rank_grads(n, N, step=t, block=23) for t in range(1, T + 1)]
+    r = oracle.Range.fresh(th0)
+    p = torch.nn.Parameter(torch.from_numpy(th0.astype(np.float64)))
+    opt = torch.optim.AdamW([p], lr=1e-3, weight_decay=1e-2, foreach=False)
+    for t, gq in enumerate(steps, start=1):
+        S, coef = oracle.adam_step_dp([r], [gq], 1.0 / N, oracle.hparams(step=t), max_grad_norm=clip)
+        mean = sum(torch.from_numpy(synth.bf16_bits_to_f32(g).astype(np.float64)) for g in gq) / N
+        p.grad = mean
+        if clip > 0:
+            tn = float(torch.nn.utils.clip_grad_norm_([p], clip, foreach=False))
+            assert abs(math.sqrt(S) - tn) <= n * 2.0 ** -53 * tn
+            assert coef < 1.0
+        opt.step()
+        with torch.no_grad():
+            p.copy_(p.float().double())
+            st = opt.state[p]
+            st["exp_avg"].copy_(st["exp_avg"].float().double())
+            st["exp_avg_sq"].copy_(st["exp_avg_sq"].float().double())
+    st = opt.state[p]
+    tp = p.detach().float().numpy()
+    check_range(dict(p32=tp, m32=st["exp_avg"].float().numpy(), v32=st["exp_avg_sq"].float().numpy(),
+                     p16=oracle.bf16_rne(tp)), r, tol=1e-6, what="dp torch")
+
+
+def test_dp_sumsq_exact_small():
+    from fractions import Fraction
+    gd = oracle.reduce_grads(_rank_grads(2000, 3, block=24), 1.0 / 3.0)
+    exact = sum(Fraction(float(x)) ** 2 for x in gd)
+    # each square and each partial sum rounds once: |err| <= 2n * 2^-53 * S
+    assert abs(Fraction(oracle.grad_sumsq_d(gd)) - exact) <= Fraction(2 * gd.size, 2 ** 53) * exact
