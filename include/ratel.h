@@ -178,6 +178,28 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
  * steps only.  The pointers are borrowed like all registered memory. */
 int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_params, int n);
 
+/* Fused data-parallel gradient reduction (reduce-scatter folded into the
+ * update, reading R17 -- the paper leaves the
+ * multi-GPU gradient semantics unspecified).  rank_grads[q]
+ * (q = 0..world_size-1, world_size <= 8) is rank q's LOCAL full-range bf16
+ * gradient of range `range_idx` of block `block_id` (numel elements, as mapped
+ * into THIS process: CUDA IPC, P2P or symmetric-memory pointers; entry [rank]
+ * is ignored -- the range's own grad_bf16 is used).  From then on the update
+ * of this rank's slice uses
+ *     g[i] = fp32( grad_scale * sum_{q=0..N-1} bf16(G16_q[i]) )
+ * (fp64 sum in rank order, one rounding; grad_scale = 1/N is the DDP mean, 1
+ * the sum), also for the clip norm.  The range must have grad_is_rank_slice
+ * = 0; not for RATEL_HOST_COMPUTE blocks (RATEL_EINVAL); grad_scale finite >
+ * 0.  Synchronisation (NCCL communicator present): each hand-off adds an
+ * 8-byte allreduce on the comm stream before the block's update -- the
+ * cross-rank "all G16 of this block are complete" barrier -- and ratel_sync's
+ * barrier keeps every G16 unmodified until all ranks finished reading it;
+ * ratel_block_wait on such a block is then collective (every rank calls it
+ * for the same blocks in the same order).  With RATEL_COMM_NONE the caller
+ * provides that ordering.  Between steps only; pointers are borrowed. */
+int ratel_register_peer_grads(int block_id, int range_idx, const void* const* rank_grads, int n,
+                              double grad_scale);
+
 /* Arms optimizer step `step` (1-based t, strictly increasing across steps)
  * with the given hyperparameters (0 <= beta < 1, lr, eps, wd >= 0, finite).
  * Blocks already handed off in this step are enqueued now (deferred mode);

@@ -212,18 +212,15 @@ __device__ __forceinline__ void load8(Frag8& f, const RangeDesc& R, uint64_t i) 
   ld_f8(R.v + 8 * i, f.v);
 }
 
+// Update octet i of R from the fp32 gradients g[0..7] (f.g unused) and
+// store theta, m, v, P16 (and the peer P16 copies).
 template <int MODE, bool CLIP>
-__device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint64_t i,
-                                              const AdamScalars& s, float coef_f, double coef_d,
-                                              const PeerDesc& pd) {
-  const uint32_t gw[4] = {f.g.x, f.g.y, f.g.z, f.g.w};
+__device__ __forceinline__ void update_store8_g(const float (&g)[8], Frag8& f, const RangeDesc& R, uint64_t i,
+                                                const AdamScalars& s, float coef_f, double coef_d,
+                                                const PeerDesc& pd) {
   const bool wd = R.wd_on != 0;
 #pragma unroll
-  for (int k = 0; k < 8; ++k) {
-    const uint32_t w = gw[k >> 1];
-    float g = bf16_bits_to_f32((k & 1) ? (w >> 16) : (w & 0xFFFFu));
-    adam_update<MODE, CLIP>(g, f.t[k], f.m[k], f.v[k], s, wd, coef_f, coef_d);
-  }
+  for (int k = 0; k < 8; ++k) adam_update<MODE, CLIP>(g[k], f.t[k], f.m[k], f.v[k], s, wd, coef_f, coef_d);
   st_f8(R.th + 8 * i, f.t);
   st_f8(R.m + 8 * i, f.m);
   st_f8(R.v + 8 * i, f.v);
@@ -234,6 +231,20 @@ __device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint
   pk.w = pack_bf16x2_rn(f.t[6], f.t[7]);
   st_p8(R.p + 8 * i, pk);
   st_peers8(pd, 8 * i, pk);
+}
+
+template <int MODE, bool CLIP>
+__device__ __forceinline__ void update_store8(Frag8& f, const RangeDesc& R, uint64_t i,
+                                              const AdamScalars& s, float coef_f, double coef_d,
+                                              const PeerDesc& pd) {
+  const uint32_t gw[4] = {f.g.x, f.g.y, f.g.z, f.g.w};
+  float g[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) {
+    const uint32_t w = gw[k >> 1];
+    g[k] = bf16_bits_to_f32((k & 1) ? (w >> 16) : (w & 0xFFFFu));
+  }
+  update_store8_g<MODE, CLIP>(g, f, R, i, s, coef_f, coef_d, pd);
 }
 
 template <int MODE, bool CLIP>
@@ -544,6 +555,99 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
   }
 }
 
+// ---- K1-RS: the data-parallel gradient reduction fused into the update ------
+// (R17).  Each rank keeps its local full-range G16;
+// for its own slice the kernel loads the N ranks' bf16 octets (the peers'
+// over NVLink, P2P), sums them in fp64 in rank order, scales once and rounds
+// once to fp32, then runs the same adam_update().  This replaces the
+// reduce-scatter: no reduced-gradient buffer, no separate NCCL kernel.  A
+// range without peer grads is the n = 1, scale = 1 case, which reproduces
+// the plain path bit for bit (fp32(1.0 * bf16) == bf16).  Register-staged
+// (LDG) like adam_update_kernel: on a real multi-GPU system the kernel is
+// bound by the 2(N-1)/N B/param of NVLink reads, not by HBM.
+constexpr int kMaxRanks = 8;
+struct GradPeers {
+  const uint16_t* g[kMaxRanks];  // every rank's G16, offset to this slice/tile, rank order
+  int n;                          // ranks summed (>= 1)
+  int pad_;
+  double scale;                   // 1/N = data-parallel mean, 1 = sum
+};
+struct RsUpdateParams {
+  UpdateParams u;
+  GradPeers gp[kMaxRanges];
+};
+struct RsSumsqParams {
+  GradPeers gp[kMaxRanges];
+  uint64_t n[kMaxRanges];
+  int nr;
+  double* partials;  // one slot per CTA
+};
+
+__device__ __forceinline__ void reduce_g8(const GradPeers& gp, uint64_t e, float (&g)[8]) {
+  uint4 w[kMaxRanks];
+#pragma unroll
+  for (int q = 0; q < kMaxRanks; ++q)
+    if (q < gp.n) w[q] = *reinterpret_cast<const uint4*>(gp.g[q] + e);
+  double s[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) s[k] = 0.0;
+#pragma unroll
+  for (int q = 0; q < kMaxRanks; ++q) {
+    if (q < gp.n) {
+      const uint32_t ws[4] = {w[q].x, w[q].y, w[q].z, w[q].w};
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        s[2 * k] = __dadd_rn(s[2 * k], static_cast<double>(bf16_bits_to_f32(ws[k] & 0xFFFFu)));
+        s[2 * k + 1] = __dadd_rn(s[2 * k + 1], static_cast<double>(bf16_bits_to_f32(ws[k] >> 16)));
+      }
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < 8; ++k) g[k] = __double2float_rn(__dmul_rn(s[k], gp.scale));
+}
+
+__device__ __forceinline__ float reduce_g1(const GradPeers& gp, uint64_t j) {
+  double s = 0.0;
+  for (int q = 0; q < gp.n; ++q) s = __dadd_rn(s, static_cast<double>(bf16_bits_to_f32(gp.g[q][j])));
+  return __double2float_rn(__dmul_rn(s, gp.scale));
+}
+
+template <int MODE, bool CLIP>
+__global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_rs_kernel(const __grid_constant__ RsUpdateParams Q) {
+  const UpdateParams& P = Q.u;
+  const double coef_d = CLIP ? clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag) : 1.0;
+  const float coef_f = static_cast<float>(coef_d);
+  const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  for (int r = 0; r < P.nr; ++r) {
+    const RangeDesc& R = P.r[r];
+    const GradPeers& gp = Q.gp[r];
+    const uint64_t n8 = R.n >> 3;
+    for (uint64_t i = tid; i < n8; i += stride) {
+      Frag8 f;
+      ld_f8(R.th + 8 * i, f.t);
+      ld_f8(R.m + 8 * i, f.m);
+      ld_f8(R.v + 8 * i, f.v);
+      float g[8];
+      reduce_g8(gp, 8 * i, g);
+      update_store8_g<MODE, CLIP>(g, f, R, i, P.s, coef_f, coef_d, P.peers[r]);
+    }
+    const uint64_t j = (n8 << 3) + tid;
+    if (j < R.n) {
+      float th = R.th[j], m = R.m[j], v = R.v[j];
+      adam_update<MODE, CLIP>(reduce_g1(gp, j), th, m, v, P.s, R.wd_on != 0, coef_f, coef_d);
+      R.th[j] = th;
+      R.m[j] = m;
+      R.v[j] = v;
+      const uint16_t pb = static_cast<uint16_t>(pack_bf16x2_rn(th, 0.0f) & 0xFFFFu);
+      R.p[j] = pb;
+      const PeerDesc& pd = P.peers[r];
+      for (int q = 0; q < pd.n; ++q) pd.p[q][j] = pb;
+    }
+  }
+  if (P.any_peers) __threadfence_system();
+}
+
 __device__ __forceinline__ double warp_sum(double x) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);
@@ -605,6 +709,34 @@ __global__ void __launch_bounds__(kThreads) grad_sumsq_kernel(const __grid_const
     }
   }
   const double t = block_sum((a0 + a1) + (a2 + a3));
+  if (threadIdx.x == 0) P.partials[blockIdx.x] = t;
+}
+
+// K2-RS.  Per-CTA partial of sum(g^2) of the REDUCED gradient (the fp32 g
+// the update uses), for the clip with the fused reduction.
+__global__ void __launch_bounds__(kThreads) grad_sumsq_rs_kernel(const __grid_constant__ RsSumsqParams P) {
+  const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  double a0 = 0.0, a1 = 0.0;
+  for (int r = 0; r < P.nr; ++r) {
+    const GradPeers& gp = P.gp[r];
+    const uint64_t n = P.n[r], n8 = n >> 3;
+    for (uint64_t i = tid; i < n8; i += stride) {
+      float g[8];
+      reduce_g8(gp, 8 * i, g);
+#pragma unroll
+      for (int k = 0; k < 8; k += 2) {
+        a0 += static_cast<double>(g[k]) * static_cast<double>(g[k]);
+        a1 += static_cast<double>(g[k + 1]) * static_cast<double>(g[k + 1]);
+      }
+    }
+    const uint64_t j = (n8 << 3) + tid;
+    if (j < n) {
+      const double x = static_cast<double>(reduce_g1(gp, j));
+      a0 += x * x;
+    }
+  }
+  const double t = block_sum(a0 + a1);
   if (threadIdx.x == 0) P.partials[blockIdx.x] = t;
 }
 

@@ -74,6 +74,13 @@ struct Block {
   cudaEvent_t ev_gh = nullptr;    // HOST_COMPUTE: G16 slices landed in host staging
   std::vector<uint16_t*> h_g, h_p;  // HOST_COMPUTE: pinned G16 / P16 staging per range (rank slice)
   std::vector<std::vector<uint16_t*>> peers;  // per range: every rank's P16 base as mapped here (fused all-gather)
+  // Fused data-parallel gradient reduction (R17): per range, every rank's
+  // full-range G16 base as mapped here (empty = plain rank-slice gradient).
+  std::vector<std::vector<const uint16_t*>> rgrads;
+  std::vector<double> rscale;
+  bool rs = false;                  // some range of this block has peer grads
+  cudaEvent_t ev_ready = nullptr;   // RS + NCCL: every rank's G16 of this block is complete
+  cudaEvent_t ev_rel = nullptr;     // RS + NCCL: every rank finished reading this block's G16
   bool handed_off = false, enqueued = false;
 };
 
@@ -95,7 +102,7 @@ struct Ctx {
   char sticky_msg[1024] = "";
   int device = 0, rank = 0, world = 1;
   ratel_config cfg{};
-  int sms = 0, k1_grid = 0, k2_grid = 0;
+  int sms = 0, k1_grid = 0, k2_grid = 0, rs_grid = 0;
   cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr, s_host = nullptr,
                s_tile = nullptr;
   cudaEvent_t ev_end[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
@@ -115,6 +122,7 @@ struct Ctx {
   double* d_sumsq = nullptr;  // [0] this rank, [1] all ranks, [2] barrier scratch
   double* d_barrier = nullptr;
   int n_peer_ranges = 0;      // ranges using the fused (peer-store) all-gather
+  int n_rs_blocks = 0;        // blocks using the fused gradient reduction
   int* h_flag = nullptr;      // mapped pinned: non-finite norm seen
   int* d_flag = nullptr;
   // pinned-host tile ring
@@ -218,7 +226,14 @@ cudaError_t prepare_k1() {
 #endif
 }
 
-int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* pd = nullptr) {
+template <int MODE, bool CLIP>
+void launch_k1_rs(const RsUpdateParams& Q, unsigned grid, cudaStream_t st) {
+  adam_update_rs_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(Q);
+}
+
+// gp != nullptr: the fused-reduction kernel (gp[i] = the rank grads of rd[i]).
+int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* pd = nullptr,
+                  const GradPeers* gp = nullptr) {
   if (nr == 0) return RATEL_OK;
   UpdateParams P{};
   uint64_t max8 = 0;
@@ -237,7 +252,8 @@ int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* 
   P.max_norm = G.cfg.max_grad_norm;
   P.nonfinite_flag = G.d_flag;
   const uint64_t want = std::max<uint64_t>(1, (max8 + kThreads - 1) / kThreads);
-  const unsigned grid = static_cast<unsigned>(std::min<uint64_t>(want, static_cast<uint64_t>(G.k1_grid)));
+  const unsigned grid = static_cast<unsigned>(
+      std::min<uint64_t>(want, static_cast<uint64_t>(gp != nullptr ? G.rs_grid : G.k1_grid)));
   TimingPair* tp = nullptr;
   if (G.cfg.timing) {
     if (G.tused == G.tpool.size()) {
@@ -249,17 +265,66 @@ int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* 
     tp = &G.tpool[G.tused++];
     CK(cudaEventRecord(tp->a, st));
   }
-  if (G.cfg.mode == RATEL_ADAMW)
+  if (gp != nullptr) {
+    static RsUpdateParams Q;  // 6.5 KB: static, not on the host stack (the API is not reentrant)
+    Q = RsUpdateParams{};
+    Q.u = P;
+    for (int i = 0; i < nr; ++i) Q.gp[i] = gp[i];
+    if (G.cfg.mode == RATEL_ADAMW)
+      clip ? launch_k1_rs<RATEL_ADAMW, true>(Q, grid, st) : launch_k1_rs<RATEL_ADAMW, false>(Q, grid, st);
+    else
+      clip ? launch_k1_rs<RATEL_ADAM_L2, true>(Q, grid, st) : launch_k1_rs<RATEL_ADAM_L2, false>(Q, grid, st);
+  } else if (G.cfg.mode == RATEL_ADAMW) {
     clip ? launch_k1<RATEL_ADAMW, true>(P, grid, st) : launch_k1<RATEL_ADAMW, false>(P, grid, st);
-  else
+  } else {
     clip ? launch_k1<RATEL_ADAM_L2, true>(P, grid, st) : launch_k1<RATEL_ADAM_L2, false>(P, grid, st);
+  }
   CK(cudaGetLastError());
   ++G.launches;
   if (tp) CK(cudaEventRecord(tp->b, st));
   return RATEL_OK;
 }
 
+// Rank grads of range i of B at element `off` of this rank's slice: every
+// rank's G16 for a range with peer grads, else this rank's own (n = 1,
+// scale = 1, which the fused kernels reduce to the plain gradient bit for bit).
+GradPeers grad_peers(const Block& B, size_t i, uint64_t off) {
+  GradPeers d{};
+  const Slice& s = B.slices[i];
+  if (i < B.rgrads.size() && !B.rgrads[i].empty()) {
+    for (int q = 0; q < G.world; ++q) {
+      const uint16_t* base = q == G.rank ? static_cast<const uint16_t*>(B.ranges[i].grad_bf16) : B.rgrads[i][q];
+      d.g[q] = base + s.begin + off;
+    }
+    d.n = G.world;
+    d.scale = B.rscale[i];
+  } else {
+    d.g[0] = grad_ptr(B.ranges[i], s) + off;
+    d.n = 1;
+    d.scale = 1.0;
+  }
+  return d;
+}
+
 int launch_sumsq(const Block& B) {
+  if (B.rs) {
+    static RsSumsqParams S;
+    S = RsSumsqParams{};
+    int nr = 0;
+    for (size_t i = 0; i < B.ranges.size(); ++i) {
+      const Slice& s = B.slices[i];
+      if (s.end == s.begin) continue;
+      S.gp[nr] = grad_peers(B, i, 0);
+      S.n[nr] = s.end - s.begin;
+      ++nr;
+    }
+    S.nr = nr;
+    S.partials = G.d_partials + static_cast<size_t>(B.order) * G.k2_grid;
+    grad_sumsq_rs_kernel<<<G.k2_grid, kThreads, 0, G.s_opt>>>(S);
+    CK(cudaGetLastError());
+    ++G.launches;
+    return RATEL_OK;
+  }
   SumsqParams S{};
   int nr = 0;
   for (size_t i = 0; i < B.ranges.size(); ++i) {
@@ -311,6 +376,8 @@ int stage_tile(const Block& B, size_t ri, uint64_t off, uint64_t len) {
   rd.p = static_cast<uint16_t*>(r.param_bf16) + s.begin + off;
   rd.n = len;
   rd.wd_on = r.apply_weight_decay != 0;
+  GradPeers gp{};
+  if (B.rs) gp = grad_peers(B, ri, off);
   const bool serial = G.cfg.staging == RATEL_STAGING_SERIALIZED;
   cudaStream_t in = serial ? G.s_tile : G.s_h2d;
   cudaStream_t out = serial ? G.s_tile : G.s_d2h;
@@ -324,7 +391,7 @@ int stage_tile(const Block& B, size_t ri, uint64_t off, uint64_t len) {
     CK(cudaStreamWaitEvent(G.s_tile, G.ev_h2d[k], 0));
   }
   const PeerDesc pd = peer_desc(B, ri, off);
-  RK(launch_update(&rd, 1, G.s_tile, &pd));
+  RK(launch_update(&rd, 1, G.s_tile, &pd, B.rs ? &gp : nullptr));
   if (!serial) {
     CK(cudaEventRecord(G.ev_k1[k], G.s_tile));
     CK(cudaStreamWaitEvent(out, G.ev_k1[k], 0));
@@ -432,11 +499,13 @@ int enqueue_block(Block& B) {
   if (B.residency == RATEL_DEVICE) {
     RangeDesc rd[kMaxRanges];
     PeerDesc pd[kMaxRanges];
+    GradPeers gp[kMaxRanges];
     int nr = 0;
     for (size_t i = 0; i < B.ranges.size(); ++i) {
       const ratel_range& r = B.ranges[i];
       const Slice& s = B.slices[i];
       if (s.end == s.begin) continue;
+      if (B.rs) gp[nr] = grad_peers(B, i, 0);
       pd[nr] = peer_desc(B, i, 0);
       RangeDesc& d = rd[nr++];
       d.g = grad_ptr(r, s);
@@ -448,11 +517,12 @@ int enqueue_block(Block& B) {
       d.wd_on = r.apply_weight_decay != 0;
       d.pad_ = 0;
     }
-    RK(launch_update(rd, nr, G.s_opt, pd));
+    RK(launch_update(rd, nr, G.s_opt, pd, B.rs ? gp : nullptr));
   } else if (B.residency == RATEL_PINNED_HOST) {
     // Tile updates run on a HIGH-priority stream: each is short and gates the
     // copy pipeline, so when a backward GEMM frees SMs they must go first.
     CK(cudaStreamWaitEvent(G.s_tile, B.ev_grad, 0));
+    if (B.rs && G.comm != nullptr) CK(cudaStreamWaitEvent(G.s_tile, B.ev_ready, 0));
     if (G.cfg.max_grad_norm > 0.0) CK(cudaStreamWaitEvent(G.s_tile, G.ev_norm, 0));
     for (size_t i = 0; i < B.ranges.size(); ++i) {
       const Slice& s = B.slices[i];
@@ -546,6 +616,8 @@ void destroy_all() {
     if (B.ev_grad) cudaEventDestroy(B.ev_grad);
     if (B.ev_done) cudaEventDestroy(B.ev_done);
     if (B.ev_gh) cudaEventDestroy(B.ev_gh);
+    if (B.ev_ready) cudaEventDestroy(B.ev_ready);
+    if (B.ev_rel) cudaEventDestroy(B.ev_rel);
     for (uint16_t* p : B.h_g) cudaFreeHost(p);
     for (uint16_t* p : B.h_p) cudaFreeHost(p);
   }
@@ -606,6 +678,13 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   else
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, adam_update_kernel<RATEL_ADAM_L2, false>, kThreads, 0));
   G.k1_grid = G.sms * std::max(occ, 1);
+  int occ_rs = 0;
+  if (c.mode == RATEL_ADAMW)
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_rs, adam_update_rs_kernel<RATEL_ADAMW, false>, kThreads, 0));
+  else
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_rs, adam_update_rs_kernel<RATEL_ADAM_L2, false>, kThreads, 0));
+  G.rs_grid = G.sms * std::max(occ_rs, 1);
+  if (c.max_ctas > 0) G.rs_grid = std::min(G.rs_grid, c.max_ctas);
   CK((prepare_k1<RATEL_ADAMW, false>()));
   CK((prepare_k1<RATEL_ADAMW, true>()));
   CK((prepare_k1<RATEL_ADAM_L2, false>()));
@@ -811,6 +890,46 @@ int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_pa
   return RATEL_OK;
 }
 
+int ratel_register_peer_grads(int block_id, int range_idx, const void* const* rank_grads, int n,
+                              double grad_scale) {
+  RK(entry());
+  if (G.armed || G.n_handed > 0) return set_error(RATEL_ESTATE, "ratel_register_peer_grads: a step is in flight");
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: block %d is not registered", block_id);
+  Block& B = G.blocks[block_id];
+  if (range_idx < 0 || range_idx >= static_cast<int>(B.ranges.size()))
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: range %d out of range", range_idx);
+  if (B.residency == RATEL_HOST_COMPUTE)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: not for HOST_COMPUTE blocks");
+  if (B.ranges[range_idx].grad_is_rank_slice)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: the range's grad must be full-range (grad_is_rank_slice = 0)");
+  if (rank_grads == nullptr || n != G.world || G.world > kMaxRanks)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: need world_size (%d <= %d) pointers", G.world,
+                     kMaxRanks);
+  if (!(grad_scale > 0.0) || !std::isfinite(grad_scale))
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: grad_scale must be finite and > 0");
+  std::vector<const uint16_t*> v(n, nullptr);
+  for (int q = 0; q < n; ++q) {
+    if (q == G.rank) continue;  // this rank's own grad_bf16 is used
+    if (rank_grads[q] == nullptr || !aligned16(rank_grads[q]))
+      return set_error(RATEL_EINVAL, "ratel_register_peer_grads: rank %d's pointer must be non-NULL, 16-byte aligned", q);
+    v[q] = static_cast<const uint16_t*>(rank_grads[q]);
+  }
+  if (G.comm != nullptr && B.ev_ready == nullptr) {
+    CK(cudaEventCreateWithFlags(&B.ev_ready, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&B.ev_rel, cudaEventDisableTiming));
+  }
+  if (B.rgrads.size() != B.ranges.size()) {
+    B.rgrads.resize(B.ranges.size());
+    B.rscale.assign(B.ranges.size(), 1.0);
+  }
+  B.rgrads[range_idx] = v;
+  B.rscale[range_idx] = grad_scale;
+  if (!B.rs) ++G.n_rs_blocks;
+  B.rs = true;
+  return RATEL_OK;
+}
+
 int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay, int64_t step) {
   Nvtx nv("ratel_adam_step %lld", static_cast<long long>(step));
   RK(entry());
@@ -870,6 +989,15 @@ int ratel_offload_grad_chunk(int block_id, void* stream) {
     return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d already handed off this step", block_id);
   CK(cudaEventRecord(B.ev_grad, static_cast<cudaStream_t>(stream)));
   CK(cudaStreamWaitEvent(G.s_opt, B.ev_grad, 0));
+  if (B.rs && G.comm != nullptr) {
+    // Fused reduction: this rank is about to read every rank's G16 of the
+    // block.  An 8-byte allreduce after the local hand-off is the barrier --
+    // once it completes, every rank's backward has produced the block.
+    CK(cudaStreamWaitEvent(G.s_comm, B.ev_grad, 0));
+    NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
+    CK(cudaEventRecord(B.ev_ready, G.s_comm));
+    CK(cudaStreamWaitEvent(G.s_opt, B.ev_ready, 0));
+  }
   B.handed_off = true;
   ++G.n_handed;
   if (G.cfg.max_grad_norm > 0.0) {
@@ -891,6 +1019,15 @@ int ratel_block_wait(int block_id, void* stream) {
   const Block& B = G.blocks[block_id];
   if (B.handed_off && !B.enqueued)
     return set_error(RATEL_ESTATE, "ratel_block_wait: block %d's update is not enqueued yet", block_id);
+  if (B.rs && G.comm != nullptr && B.enqueued) {
+    // Peers read this rank's G16 too: release it only after every rank's
+    // update of the block (collective: every rank calls block_wait alike).
+    CK(cudaStreamWaitEvent(G.s_comm, B.ev_done, 0));
+    NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
+    CK(cudaEventRecord(B.ev_rel, G.s_comm));
+    CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), B.ev_rel, 0));
+    return RATEL_OK;
+  }
   CK(cudaStreamWaitEvent(static_cast<cudaStream_t>(stream), B.ev_done, 0));
   return RATEL_OK;
 }
@@ -903,11 +1040,12 @@ int ratel_sync(void* stream) {
     if (G.n_handed != static_cast<int>(G.reg.size()))
       return set_error(RATEL_ESTATE, "ratel_sync: %d of %zu blocks handed off", G.n_handed, G.reg.size());
   }
-  if (G.comm != nullptr && G.n_peer_ranges > 0) {
-    // Fused all-gather: ranks wrote into each other's P16.  One 8-byte
-    // allreduce after every local update is the cross-rank barrier: once it
-    // completes here, every rank's update kernels (and their peer stores,
-    // fenced system-wide) have finished.
+  if (G.comm != nullptr && (G.n_peer_ranges > 0 || G.n_rs_blocks > 0)) {
+    // Fused all-gather: ranks wrote into each other's P16; fused reduction:
+    // ranks read each other's G16.  One 8-byte allreduce after every local
+    // update is the cross-rank barrier: once it completes here, every rank's
+    // update kernels (their peer stores fenced system-wide, their peer loads
+    // done) have finished.
     CK(cudaEventRecord(G.ev_end[0], G.s_opt));
     CK(cudaEventRecord(G.ev_end[5], G.s_tile));
     CK(cudaStreamWaitEvent(G.s_comm, G.ev_end[0], 0));

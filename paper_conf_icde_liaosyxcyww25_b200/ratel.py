@@ -92,6 +92,7 @@ def load_library(path: str = _LIB_PATH, strict: bool = True):
         "ratel_sync": (I, [P]),
         "ratel_block_wait": (I, [I, P]),
         "ratel_register_peer_params": (I, [I, I, ctypes.POINTER(P), I]),
+        "ratel_register_peer_grads": (I, [I, I, ctypes.POINTER(P), I, D]),
         "ratel_finalize": (I, []),
         "ratel_last_error": (ctypes.c_char_p, []),
         "ratel_padded_numel": (U64, [U64, I]),
@@ -172,6 +173,14 @@ def ratel_register_peer_params(block_id: int, range_idx: int, peer_params) -> No
     ptrs = [(p.data_ptr() if hasattr(p, "data_ptr") else (int(p) if p else None)) for p in peer_params]
     arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
     _check(_lib.ratel_register_peer_params(block_id, range_idx, arr, len(ptrs)))
+
+
+def ratel_register_peer_grads(block_id: int, range_idx: int, rank_grads, grad_scale: float) -> None:
+    """rank_grads: every rank's full-range G16 of the range (int, tensor or
+    None for this rank), rank order; grad_scale 1/N = data-parallel mean."""
+    ptrs = [(p.data_ptr() if hasattr(p, "data_ptr") else (int(p) if p else None)) for p in rank_grads]
+    arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
+    _check(_lib.ratel_register_peer_grads(block_id, range_idx, arr, len(ptrs), grad_scale))
 
 
 def ratel_adam_step(lr: float, beta1: float, beta2: float, eps: float, weight_decay: float, step: int) -> None:
