@@ -208,7 +208,7 @@ def workload_config(args, world):
             "parallelism": (f"range-sharded x{world}" + (" (fused peer-store all-gather)" if args.fused_allgather else
                                                           " (NCCL all-gather)")) if world > 1 else "single GPU",
             "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
-            "max_grad_norm": args.clip}
+            "max_grad_norm": args.clip, "update_streams": args.update_streams}
 
 
 class PinnedArena:
@@ -653,6 +653,8 @@ def main():
                     help="arm before the hand-offs (AGO) or after the last one (deferred)")
     ap.add_argument("--tile-elems", type=int, default=0)
     ap.add_argument("--depth", type=int, default=0)
+    ap.add_argument("--update-streams", type=int, default=2, choices=[1, 2],
+                    help="device-residency update kernels alternate over this many streams")
     args = ap.parse_args()
     global ARM_AFTER
     ARM_AFTER = args.arm == "after"
@@ -701,6 +703,7 @@ def main():
     if args.depth:
         cfg.pipeline_depth = args.depth
     cfg.host_threads = args.host_threads
+    cfg.update_streams = args.update_streams
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
     try:

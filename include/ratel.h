@@ -114,6 +114,9 @@ typedef struct {
   int timing;             /* 1: bracket every update-kernel launch with CUDA events (ratel_kernel_timing) */
   int comm;               /* ratel_comm; default RATEL_COMM_AUTO */
   int host_threads;       /* HOST_COMPUTE handler threads (0 = OpenMP default: all cores) */
+  int update_streams;     /* device-residency updates alternate over this many low-priority streams,
+                             1..2; default 2: block b+1's update starts on the SMs block b's tail
+                             frees instead of after it (results are identical) */
 } ratel_config;
 
 /* One contiguous parameter range of a block (a flat tensor, or a block's
@@ -266,8 +269,10 @@ int ratel_get_grad_sumsq(double* out);
 int ratel_alloc_pinned(uint64_t bytes, void** out);
 int ratel_free_pinned(void* p);
 
-/* Sum of the update kernel's event-timed durations (ms) and number of timed
- * launches since the last reset (requires cfg.timing = 1; blocking). */
+/* Busy time of the update kernels (ms) -- the union of the event-timed
+ * [start, end] intervals of every launch, so overlapping launches on the two
+ * update streams are not double counted -- and the number of timed launches
+ * since the last reset (requires cfg.timing = 1; blocking). */
 int ratel_kernel_timing(double* total_ms, int64_t* launches, int reset);
 
 /* Number of kernels this library launched since init (update, grad-norm

@@ -71,6 +71,11 @@ struct UpdateParams {
   const double* sumsq;   // clip: global sum of g^2 (device); unused otherwise
   double max_norm;
   int* nonfinite_flag;   // clip: set to !isfinite(sumsq) by CTA 0
+  // TMA kernel tile scheduler: NULL = static round robin; else tiles are
+  // taken dynamically, tile = atomicAdd(tile_ctr, 1) - tile_base (the
+  // counter only grows; one launch advances it by tiles + grid).
+  unsigned long long* tile_ctr;
+  unsigned long long tile_base;
 };
 
 struct SumsqParams {
@@ -340,7 +345,7 @@ constexpr int kTmaThreads = 32 * (kTmaConsumerWarps + 1);
 constexpr int kTmaTile = kTmaConsumerWarps * 32 * 8;          // elements per tile (1 octet per consumer thread)
 constexpr int kTmaStages = RATEL_TMA_STAGES;
 constexpr uint32_t kTmaStageBytes = kTmaTile * 14;            // g 2 + theta/m/v 12
-constexpr uint32_t kTmaSmemBytes = kTmaStages * kTmaStageBytes + 2 * kTmaStages * 8;
+constexpr uint32_t kTmaSmemBytes = kTmaStages * kTmaStageBytes + 3 * kTmaStages * 8;  // + full/empty/tile id
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -412,6 +417,7 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
   extern __shared__ __align__(128) uint8_t smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kTmaStages * kTmaStageBytes);
   uint64_t* empty = full + kTmaStages;
+  volatile uint64_t* tile_id = empty + kTmaStages;  // the producer's tile per stage (~0 = no more)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kTmaStages; ++s) {
@@ -428,12 +434,26 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
 
   if (warp == kTmaConsumerWarps) {  // producer
     if (lane == 0) {
+      // Dynamic scheduling: CTAs that run ahead take more tiles, so all SMs
+      // finish together (a static split left the slowest SM's tail exposed;
+      // measured in DESIGN.md §6).  The next grab is issued one tile early so
+      // its latency overlaps the wait for a free stage.
+      const bool dyn = P.tile_ctr != nullptr;
+      uint64_t k = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : blockIdx.x;
       int stage = 0;
       uint32_t phase = 0;
-      for (uint64_t k = blockIdx.x; k < total; k += gridDim.x) {
+      for (;;) {
+        uint64_t kn = k;
+        if (k < total) kn = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : k + gridDim.x;
+        mbar_wait(&empty[stage], phase ^ 1);
+        if (k >= total) {  // no more tiles: tell the consumers
+          tile_id[stage] = ~0ull;
+          mbar_arrive(&full[stage]);
+          break;
+        }
+        tile_id[stage] = k;
         const TileLoc t = locate_tile(P, k);
         const RangeDesc& R = P.r[t.r];
-        mbar_wait(&empty[stage], phase ^ 1);
         uint8_t* base = smem + stage * kTmaStageBytes;
         mbar_expect_tx(&full[stage], t.len * 14u);
         bulk_load(base, R.g + t.off, t.len * 2u, &full[stage]);
@@ -444,6 +464,7 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
           stage = 0;
           phase ^= 1;
         }
+        k = kn;
       }
     }
   } else {  // consumers
@@ -454,10 +475,12 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
     int prev_stage = -1;
     (void)prev_stage;
     const uint32_t o = threadIdx.x;  // octet within the tile
-    for (uint64_t k = blockIdx.x; k < total; k += gridDim.x) {
+    for (;;) {
+      mbar_wait(&full[stage], phase);
+      const uint64_t k = tile_id[stage];
+      if (k == ~0ull) break;
       const TileLoc t = locate_tile(P, k);
       const RangeDesc& R = P.r[t.r];
-      mbar_wait(&full[stage], phase);
       const uint8_t* base = smem + stage * kTmaStageBytes;
       const bool valid = 8 * o < t.len;
       Frag8 f;

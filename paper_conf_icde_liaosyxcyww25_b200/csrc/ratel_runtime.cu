@@ -105,7 +105,12 @@ struct Ctx {
   int sms = 0, k1_grid = 0, k2_grid = 0, rs_grid = 0;
   cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr, s_host = nullptr,
                s_tile = nullptr;
-  cudaEvent_t ev_end[6] = {nullptr, nullptr, nullptr, nullptr, nullptr, nullptr};
+  // Device-residency update kernels alternate over s_k[0..update_streams-1];
+  // s_opt joins each (ev_done) so it stays ordered after every grad read.
+  cudaStream_t s_k[2] = {nullptr, nullptr};
+  unsigned k_next = 0;
+  static constexpr int kNS = 8;  // every stream, for the sync cross-waits
+  cudaEvent_t ev_end[kNS] = {};
   cudaEvent_t ev_norm = nullptr;  // clip: global norm final (on s_opt)
   double* h_sumsq = nullptr;      // clip + HOST_COMPUTE: pinned copy of the norm
   double hp_lr = 0, hp_b1 = 0, hp_b2 = 0, hp_eps = 0, hp_wd = 0, hp_bc1 = 1, hp_bc2 = 1;
@@ -121,6 +126,11 @@ struct Ctx {
   size_t partial_cap = 0;  // slots
   double* d_sumsq = nullptr;  // [0] this rank, [1] all ranks, [2] barrier scratch
   double* d_barrier = nullptr;
+  // TMA update kernel's dynamic tile counters, one per launching stream
+  // (s_k[0], s_k[1], s_tile, s_opt): launches on one stream are serialised,
+  // so each counter's value at a launch is known on the host (ctr_base).
+  unsigned long long* d_ctr = nullptr;
+  unsigned long long ctr_base[4] = {0, 0, 0, 0};
   int n_peer_ranges = 0;      // ranges using the fused (peer-store) all-gather
   int n_rs_blocks = 0;        // blocks using the fused gradient reduction
   int* h_flag = nullptr;      // mapped pinned: non-finite norm seen
@@ -201,8 +211,16 @@ const uint16_t* grad_ptr(const ratel_range& r, const Slice& s) {
 #define RATEL_K1_TMA 1
 #endif
 
+#ifndef RATEL_TMA_DYNAMIC
+#define RATEL_TMA_DYNAMIC 1
+#endif
+
+int ctr_slot(cudaStream_t st) {
+  return st == G.s_k[0] ? 0 : st == G.s_k[1] ? 1 : st == G.s_tile ? 2 : 3;
+}
+
 template <int MODE, bool CLIP>
-void launch_k1(const UpdateParams& P, unsigned grid, cudaStream_t st) {
+void launch_k1(UpdateParams& P, unsigned grid, cudaStream_t st) {
 #if RATEL_K1_TMA
   (void)grid;
   uint64_t tiles = 0;
@@ -210,6 +228,12 @@ void launch_k1(const UpdateParams& P, unsigned grid, cudaStream_t st) {
   uint64_t cap = static_cast<uint64_t>(G.sms) * RATEL_TMA_CTAS_PER_SM;
   if (G.cfg.max_ctas > 0) cap = std::min<uint64_t>(cap, static_cast<uint64_t>(G.cfg.max_ctas));
   const unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
+#if RATEL_TMA_DYNAMIC
+  const int slot = ctr_slot(st);
+  P.tile_ctr = G.d_ctr + slot;
+  P.tile_base = G.ctr_base[slot];
+  G.ctr_base[slot] += tiles + g;  // every tile taken once + one final grab per CTA
+#endif
   adam_update_tma_kernel<MODE, CLIP><<<g, kTmaThreads, kTmaSmemBytes, st>>>(P);
 #else
   adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(P);
@@ -496,7 +520,16 @@ int enqueue_host_compute(Block& B) {
 // hand-off).  Device residency: one K1 launch over the rank's slices of all
 // ranges.  Pinned-host: the tile ring.
 int enqueue_block(Block& B) {
+  cudaStream_t ks = G.s_opt;
   if (B.residency == RATEL_DEVICE) {
+    // Alternate update streams: this block's kernel can take the SMs the
+    // previous block's tail leaves idle (one CTA per SM does not co-reside).
+    if (G.cfg.update_streams > 1) {
+      ks = G.s_k[G.k_next++ & 1u];
+      CK(cudaStreamWaitEvent(ks, B.ev_grad, 0));
+      if (B.rs && G.comm != nullptr) CK(cudaStreamWaitEvent(ks, B.ev_ready, 0));
+      if (G.cfg.max_grad_norm > 0.0) CK(cudaStreamWaitEvent(ks, G.ev_norm, 0));
+    }
     RangeDesc rd[kMaxRanges];
     PeerDesc pd[kMaxRanges];
     GradPeers gp[kMaxRanges];
@@ -517,7 +550,7 @@ int enqueue_block(Block& B) {
       d.wd_on = r.apply_weight_decay != 0;
       d.pad_ = 0;
     }
-    RK(launch_update(rd, nr, G.s_opt, pd, B.rs ? gp : nullptr));
+    RK(launch_update(rd, nr, ks, pd, B.rs ? gp : nullptr));
   } else if (B.residency == RATEL_PINNED_HOST) {
     // Tile updates run on a HIGH-priority stream: each is short and gates the
     // copy pipeline, so when a backward GEMM frees SMs they must go first.
@@ -534,7 +567,8 @@ int enqueue_block(Block& B) {
   if (B.residency == RATEL_HOST_COMPUTE)
     RK(enqueue_host_compute(B));
   else
-    CK(cudaEventRecord(B.ev_done, B.residency == RATEL_PINNED_HOST ? G.s_tile : G.s_opt));
+    CK(cudaEventRecord(B.ev_done, B.residency == RATEL_PINNED_HOST ? G.s_tile : ks));
+  if (ks != G.s_opt) CK(cudaStreamWaitEvent(G.s_opt, B.ev_done, 0));
   // Keep ratel_optimizer_stream() ordered after every read of this block's
   // grad (so grad.record_stream(ratel_optimizer_stream()) stays sufficient).
   if (B.residency == RATEL_PINNED_HOST) CK(cudaStreamWaitEvent(G.s_opt, B.ev_done, 0));
@@ -597,6 +631,7 @@ int validate_config(const ratel_config& c) {
   if (c.comm != RATEL_COMM_AUTO && c.comm != RATEL_COMM_NONE && c.comm != RATEL_COMM_NCCL)
     return set_error(RATEL_EINVAL, "cfg.comm");
   if (c.host_threads < 0) return set_error(RATEL_EINVAL, "cfg.host_threads must be >= 0");
+  if (c.update_streams < 1 || c.update_streams > 2) return set_error(RATEL_EINVAL, "cfg.update_streams must be 1 or 2");
   return RATEL_OK;
 }
 
@@ -635,11 +670,12 @@ void destroy_all() {
   if (G.d_tiles) cudaFree(G.d_tiles);
   if (G.d_partials) cudaFree(G.d_partials);
   if (G.d_sumsq) cudaFree(G.d_sumsq);
+  if (G.d_ctr) cudaFree(G.d_ctr);
   if (G.h_flag) cudaFreeHost(G.h_flag);
   if (G.h_sumsq) cudaFreeHost(G.h_sumsq);
   if (G.ev_norm) cudaEventDestroy(G.ev_norm);
   if (G.comm) g_nccl.CommDestroy(G.comm);
-  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile})
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
     if (s) cudaStreamDestroy(s);
   G.~Ctx();
   new (&G) Ctx();
@@ -660,6 +696,8 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   int least = 0, greatest = 0;
   CK(cudaDeviceGetStreamPriorityRange(&least, &greatest));
   CK(cudaStreamCreateWithPriority(&G.s_opt, cudaStreamNonBlocking, least));  // lowest priority
+  CK(cudaStreamCreateWithPriority(&G.s_k[0], cudaStreamNonBlocking, least));
+  CK(cudaStreamCreateWithPriority(&G.s_k[1], cudaStreamNonBlocking, least));
   CK(cudaStreamCreateWithPriority(&G.s_h2d, cudaStreamNonBlocking, greatest));
   CK(cudaStreamCreateWithPriority(&G.s_d2h, cudaStreamNonBlocking, greatest));
   CK(cudaStreamCreateWithPriority(&G.s_comm, cudaStreamNonBlocking, greatest));
@@ -691,6 +729,8 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK((prepare_k1<RATEL_ADAM_L2, true>()));
   if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
   G.k2_grid = G.sms * 4;
+  CK(cudaMalloc(&G.d_ctr, 4 * sizeof(unsigned long long)));
+  CK(cudaMemset(G.d_ctr, 0, 4 * sizeof(unsigned long long)));
   CK(cudaMalloc(&G.d_sumsq, 3 * sizeof(double)));
   CK(cudaMemset(G.d_sumsq, 0, 3 * sizeof(double)));
   G.d_barrier = G.d_sumsq + 2;
@@ -729,6 +769,7 @@ void ratel_default_config(ratel_config* cfg) {
   cfg->timing = 0;
   cfg->comm = RATEL_COMM_AUTO;
   cfg->host_threads = 0;
+  cfg->update_streams = 2;
 }
 
 uint64_t ratel_padded_numel(uint64_t numel, int world_size) {
@@ -972,7 +1013,7 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
   // the whole backward -- every handler stream waits for every gradient
   // handed off so far before any state moves (s_opt already waited on each).
   if (!G.pending.empty())
-    for (cudaStream_t st : {G.s_h2d, G.s_d2h, G.s_host, G.s_tile})
+    for (cudaStream_t st : {G.s_h2d, G.s_d2h, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
       for (int id : G.pending) CK(cudaStreamWaitEvent(st, G.blocks[id].ev_grad, 0));
   for (int id : G.pending) RK(enqueue_block(G.blocks[id]));
   G.pending.clear();
@@ -1052,8 +1093,8 @@ int ratel_sync(void* stream) {
     CK(cudaStreamWaitEvent(G.s_comm, G.ev_end[5], 0));
     NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
   }
-  constexpr int NS = 6;
-  cudaStream_t ss[NS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile};
+  constexpr int NS = Ctx::kNS;
+  cudaStream_t ss[NS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]};
   for (int i = 0; i < NS; ++i) CK(cudaEventRecord(G.ev_end[i], ss[i]));
   // Order the internal streams too: the next step's stage-in must not read
   // host states still being written back, and its K1 must not overwrite a
@@ -1084,7 +1125,7 @@ int ratel_sync(void* stream) {
 int ratel_finalize(void) {
   if (!G.inited) return set_error(RATEL_ESTATE, "ratel_finalize: not initialised");
   cudaSetDevice(G.device);
-  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile})
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
     if (s) cudaStreamSynchronize(s);
   destroy_all();
   cudaGetLastError();
@@ -1105,13 +1146,29 @@ int ratel_get_grad_sumsq(double* out) {
 int ratel_kernel_timing(double* total_ms, int64_t* launches, int reset) {
   RK(entry());
   if (total_ms == nullptr || launches == nullptr) return set_error(RATEL_EINVAL, "ratel_kernel_timing: NULL");
-  double tot = 0.0;
+  // Union of the launch intervals, all measured from the first launch's start
+  // event (earlier events give negative offsets).
+  std::vector<std::pair<double, double>> iv;
+  iv.reserve(G.tused);
   for (size_t i = 0; i < G.tused; ++i) {
     CK(cudaEventSynchronize(G.tpool[i].b));
-    float ms = 0.f;
-    CK(cudaEventElapsedTime(&ms, G.tpool[i].a, G.tpool[i].b));
-    tot += ms;
+    float s = 0.f, e = 0.f;
+    CK(cudaEventElapsedTime(&s, G.tpool[0].a, G.tpool[i].a));
+    CK(cudaEventElapsedTime(&e, G.tpool[0].a, G.tpool[i].b));
+    iv.emplace_back(s, e);
   }
+  std::sort(iv.begin(), iv.end());
+  double tot = 0.0, cs = 0.0, ce = -1e300;
+  for (const auto& x : iv) {
+    if (x.first > ce) {
+      if (ce > cs) tot += ce - cs;
+      cs = x.first;
+      ce = x.second;
+    } else {
+      ce = std::max(ce, x.second);
+    }
+  }
+  if (!iv.empty() && ce > cs) tot += ce - cs;
   *total_ms = tot;
   *launches = static_cast<int64_t>(G.tused);
   if (reset) G.tused = 0;

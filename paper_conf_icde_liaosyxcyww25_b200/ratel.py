@@ -58,6 +58,7 @@ class ratel_config(ctypes.Structure):
         ("timing", ctypes.c_int),
         ("comm", ctypes.c_int),
         ("host_threads", ctypes.c_int),
+        ("update_streams", ctypes.c_int),
     ]
 
 

@@ -104,11 +104,13 @@ def run(nblocks=8, steps=10, warmup=3, rounds=3):
     for path in libs:
         ok = check_variant(torch, R, R.load_library(path, strict=False), ref)
         print(json.dumps({"variant": os.path.basename(path), "bitwise_equal_to_intree": ok}), flush=True)
-    for rnd, path in [(r, p) for r in range(rounds) for p in libs]:
+    uss = [int(x) for x in os.environ.get("RATEL_SWEEP_US", "1").split(",")]
+    for rnd, path, us in [(r, p, u) for r in range(rounds) for p in libs for u in uss]:
         L = R.load_library(path, strict=False)
         cfg = R.ratel_config()
         L.ratel_default_config(ctypes.byref(cfg))
         cfg.timing = 1
+        cfg.update_streams = us
         assert L.ratel_init(0, 0, 1, None, ctypes.byref(cfg)) == 0, L.ratel_last_error()
         for b, (p, th, m, v) in enumerate(blocks):
             rr = R.make_range(p, g, th, m, v, n)
@@ -136,8 +138,9 @@ def run(nblocks=8, steps=10, warmup=3, rounds=3):
         step_ms = e0.elapsed_time(e1) / steps
         bytes_ = 28 * n * nblocks * steps
         k1 = bytes_ / (ms.value / 1e3) / 1e9
-        results.setdefault(os.path.basename(path), []).append(k1)
-        print(json.dumps({"round": rnd, "variant": os.path.basename(path), "k1_gbs": k1,
+        name = os.path.basename(path) + f"/us{us}"
+        results.setdefault(name, []).append(k1)
+        print(json.dumps({"round": rnd, "variant": name, "k1_gbs": k1,
                           "step_gbs": 28 * n * nblocks / (step_ms / 1e3) / 1e9,
                           "avg_launch_ms": ms.value / cnt.value}), flush=True)
         assert L.ratel_finalize() == 0
