@@ -635,27 +635,69 @@ __device__ __forceinline__ float reduce_g1(const GradPeers& gp, uint64_t j) {
   return __double2float_rn(__dmul_rn(s, gp.scale));
 }
 
+// Tiles of kRsTile elements of the ranges' vector bodies, taken dynamically
+// from the same per-stream counter as the TMA kernel (tile = atomicAdd - base,
+// the next grab issued while the current tile is processed); each thread
+// updates kRsTile / 8 / kThreads octets of a tile.
+constexpr int kRsTile = 4096;
+static_assert(kRsTile % (8 * kThreads) == 0, "RS tile = whole octets per thread");
+
+__device__ __forceinline__ TileLoc locate_rs_tile(const UpdateParams& P, uint64_t k) {
+  TileLoc t{0, 0, 0};
+  for (int r = 0; r < P.nr; ++r) {
+    const uint64_t body = P.r[r].n & ~7ull;
+    const uint64_t nt = (body + kRsTile - 1) / kRsTile;
+    if (k < nt) {
+      t.r = r;
+      t.off = k * kRsTile;
+      t.len = static_cast<uint32_t>(body - t.off < (uint64_t)kRsTile ? body - t.off : kRsTile);
+      return t;
+    }
+    k -= nt;
+  }
+  t.r = -1;
+  return t;
+}
+
 template <int MODE, bool CLIP>
 __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_rs_kernel(const __grid_constant__ RsUpdateParams Q) {
   const UpdateParams& P = Q.u;
   const double coef_d = CLIP ? clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag) : 1.0;
   const float coef_f = static_cast<float>(coef_d);
-  const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
-  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
-  for (int r = 0; r < P.nr; ++r) {
+  uint64_t total = 0;
+  for (int r = 0; r < P.nr; ++r) total += ((P.r[r].n & ~7ull) + kRsTile - 1) / kRsTile;
+  __shared__ uint64_t s_next;
+  const bool dyn = P.tile_ctr != nullptr;
+  if (threadIdx.x == 0) s_next = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : blockIdx.x;
+  for (;;) {
+    __syncthreads();
+    const uint64_t k = s_next;
+    __syncthreads();
+    if (k >= total) break;
+    if (threadIdx.x == 0) s_next = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : k + gridDim.x;
+    const TileLoc t = locate_rs_tile(P, k);
+    const RangeDesc& R = P.r[t.r];
+    const GradPeers& gp = Q.gp[t.r];
+#pragma unroll
+    for (int u = 0; u < kRsTile / (8 * kThreads); ++u) {
+      const uint32_t o = threadIdx.x + u * kThreads;  // octet within the tile
+      if (8 * o < t.len) {
+        const uint64_t i = (t.off >> 3) + o;
+        Frag8 f;
+        ld_f8(R.th + 8 * i, f.t);
+        ld_f8(R.m + 8 * i, f.m);
+        ld_f8(R.v + 8 * i, f.v);
+        float g[8];
+        reduce_g8(gp, 8 * i, g);
+        update_store8_g<MODE, CLIP>(g, f, R, i, P.s, coef_f, coef_d, P.peers[t.r]);
+      }
+    }
+  }
+  // scalar tails (< 8 elements per range), CTA 0
+  for (int r = 0; r < P.nr && blockIdx.x == 0; ++r) {
     const RangeDesc& R = P.r[r];
     const GradPeers& gp = Q.gp[r];
-    const uint64_t n8 = R.n >> 3;
-    for (uint64_t i = tid; i < n8; i += stride) {
-      Frag8 f;
-      ld_f8(R.th + 8 * i, f.t);
-      ld_f8(R.m + 8 * i, f.m);
-      ld_f8(R.v + 8 * i, f.v);
-      float g[8];
-      reduce_g8(gp, 8 * i, g);
-      update_store8_g<MODE, CLIP>(g, f, R, i, P.s, coef_f, coef_d, P.peers[r]);
-    }
-    const uint64_t j = (n8 << 3) + tid;
+    const uint64_t j = (R.n & ~7ull) + threadIdx.x;
     if (j < R.n) {
       float th = R.th[j], m = R.m[j], v = R.v[j];
       adam_update<MODE, CLIP>(reduce_g1(gp, j), th, m, v, P.s, R.wd_on != 0, coef_f, coef_d);

@@ -251,8 +251,19 @@ cudaError_t prepare_k1() {
 }
 
 template <int MODE, bool CLIP>
-void launch_k1_rs(const RsUpdateParams& Q, unsigned grid, cudaStream_t st) {
-  adam_update_rs_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(Q);
+void launch_k1_rs(RsUpdateParams& Q, unsigned grid, cudaStream_t st) {
+  (void)grid;
+  uint64_t tiles = 0;
+  for (int r = 0; r < Q.u.nr; ++r) tiles += ((Q.u.r[r].n & ~7ull) + kRsTile - 1) / kRsTile;
+  const unsigned g = static_cast<unsigned>(
+      std::max<uint64_t>(1, std::min<uint64_t>(tiles, static_cast<uint64_t>(G.rs_grid))));
+#if RATEL_TMA_DYNAMIC
+  const int slot = ctr_slot(st);
+  Q.u.tile_ctr = G.d_ctr + slot;
+  Q.u.tile_base = G.ctr_base[slot];
+  G.ctr_base[slot] += tiles + g;
+#endif
+  adam_update_rs_kernel<MODE, CLIP><<<g, kThreads, 0, st>>>(Q);
 }
 
 // gp != nullptr: the fused-reduction kernel (gp[i] = the rank grads of rd[i]).
