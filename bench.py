@@ -70,13 +70,19 @@ def peaks():
         return 6650.0, "fallback"
 
 
-def ncu_traffic_per_param():
-    """dram bytes per param of K1 from the committed ncu summary, if any."""
+def ncu_summary():
+    """K1's committed ncu --set full summary (profiles/k1_ncu_summary.json), if any."""
     try:
         with open(os.path.join(ROOT, "profiles", "k1_ncu_summary.json")) as f:
-            return float(json.load(f)["dram_bytes_per_param"])
+            return json.load(f)
     except Exception:
-        return None
+        return {}
+
+
+def ncu_traffic_per_param():
+    """dram bytes per param of K1 from the committed ncu summary, if any."""
+    v = ncu_summary().get("dram_bytes_per_param")
+    return float(v) if v is not None else None
 
 
 class ClockSampler:
@@ -766,7 +772,9 @@ def main():
                 "algorithmic_bytes_per_launch": BYTES_PER_PARAM * per_launch,
                 "launches": k1_n, "avg_launch_ms": k1_ms / max(k1_n, 1),
                 "k1_share_of_step": (k1_ms / args.steps) / (ms / args.steps),
-                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind})"}
+                "peak_source": f"MEASURED_PEAKS.json hbm_gbs ({peak_kind}): a torch copy, whose grid-stride "
+                               "loop splits work statically; K1 schedules tiles dynamically and can exceed it",
+                "ncu_dram_pct_of_peak": ncu_summary().get("ncu_dram_pct_of_peak_sustained")}
         overlap = None
         if args.overlap_tokens > 0 and world == 1 and args.residency == "device" and args.clip == 0:
             try:

@@ -74,7 +74,8 @@ enum {
   RATEL_ECUDA = -3,      /* CUDA runtime failure (sticky) */
   RATEL_ENCCL = -4,      /* NCCL failure (sticky) */
   RATEL_ENOMEM = -5,     /* device/host allocation failed (sticky) */
-  RATEL_ENONFINITE = -6  /* clip mode: global grad norm was NaN/Inf (update still applied, like torch) */
+  RATEL_ENONFINITE = -6, /* clip mode: global grad norm was NaN/Inf (update still applied, like torch) */
+  RATEL_EIO = -7         /* SSD residency: a state file read/write failed (sticky) */
 };
 
 /* Where a block's fp32 states live and who updates them:
@@ -88,7 +89,16 @@ enum {
  *                 produces P16 (fp32 arithmetic, SIMD + OpenMP), P16 copied
  *                 host->device (2 B/param); stream-ordered via
  *                 cudaLaunchHostFunc, the host thread never blocks. */
-typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2 } ratel_residency;
+/*   SSD           the paper's storage tier (§IV-C Fig. 3b; Eq. 5
+ *                 "14P/BW_S2M + 14P/BW_M2S"): states in a file
+ *                 (ratel_register_ssd); a reader thread streams each tile
+ *                 file -> pinned staging -> device tile, the GPU kernel
+ *                 updates it, and a writer thread writes it back, so the read
+ *                 of tile k+1, the update of tile k and the write-back of
+ *                 tile k-1 overlap.  A block's reads start when its gradient
+ *                 is complete (the active message; the reader thread waits on
+ *                 the hand-off event).  Single rank (no NCCL communicator). */
+typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2, RATEL_SSD = 3 } ratel_residency;
 typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
 /* Pinned-host staging schedule: PIPELINED = Fig. 3b (stage-in of tile k+1,
  * update of tile k and write-back of tile k-1 overlap on three streams; the
@@ -202,6 +212,26 @@ int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_pa
  * provides that ordering.  Between steps only; pointers are borrowed. */
 int ratel_register_peer_grads(int block_id, int range_idx, const void* const* rank_grads, int n,
                               double grad_scale);
+
+/* SSD residency (RATEL_SSD): attach the state file of range
+ * `range_idx` of block `block_id`.  The rank slice's theta, m and v are fp32
+ * arrays in the file at `offset`, `offset + S` and `offset + 2S`, with
+ * S = ratel_ssd_range_bytes(numel, world, rank) / 3 (each array padded to a
+ * multiple of 4096 bytes; the padding is read and written back unchanged).
+ * fd: open for reading and writing (O_RDWR), borrowed until ratel_finalize;
+ * open it with O_DIRECT to bypass the page cache (the measured numbers do);
+ * offset: multiple of 4096; the file must already hold offset + 3S bytes and
+ * the initial states (the caller writes theta0, m = v = 0).  Requires
+ * cfg.tile_elems to be a multiple of 1024.  Every range of an SSD block
+ * needs a file before its first hand-off (RATEL_ESTATE otherwise).  Between
+ * steps only.  RATEL_EINVAL on a bad fd, alignment or short file.  With SSD
+ * blocks, ratel_sync (either form) also waits on the host until every state
+ * write-back of the step has reached the file. */
+int ratel_register_ssd(int block_id, int range_idx, int fd, uint64_t offset);
+
+/* Bytes one range's states take in an SSD state file (3 x 4096-padded fp32
+ * arrays of the rank's slice; 0 for an empty slice).  Pure host function. */
+uint64_t ratel_ssd_range_bytes(uint64_t numel, int world_size, int rank);
 
 /* Arms optimizer step `step` (1-based t, strictly increasing across steps)
  * with the given hyperparameters (0 <= beta < 1, lr, eps, wd >= 0, finite).

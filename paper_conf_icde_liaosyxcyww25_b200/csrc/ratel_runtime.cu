@@ -14,8 +14,19 @@
 // host link is duplex, unlike the paper's SSD link).
 #include <cuda_runtime.h>
 
+#include <fcntl.h>
+#include <sys/stat.h>
+#include <unistd.h>
+
 #include <algorithm>
+#include <atomic>
+#include <cerrno>
+#include <condition_variable>
+#include <deque>
+#include <mutex>
 #include <new>
+#include <string>
+#include <thread>
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
@@ -57,8 +68,6 @@ int set_error(int code, const char* fmt, ...) {
   return code;
 }
 
-constexpr int kMaxDepth = 16;  // pinned-host tile ring slots
-
 struct Slice {
   uint64_t begin = 0, end = 0;
 };
@@ -82,6 +91,44 @@ struct Block {
   cudaEvent_t ev_ready = nullptr;   // RS + NCCL: every rank's G16 of this block is complete
   cudaEvent_t ev_rel = nullptr;     // RS + NCCL: every rank finished reading this block's G16
   bool handed_off = false, enqueued = false;
+  // SSD residency: per range, the state file and where the slice's arrays are
+  struct SsdRange {
+    int fd = -1;
+    uint64_t off = 0, stride = 0;  // theta at off, m at off + stride, v at off + 2*stride (bytes)
+  };
+  std::vector<SsdRange> ssd;
+  uint64_t ssd_seq = 0;  // engine job number of this block's last submission
+};
+
+// The SSD tier's reader/writer threads (RATEL_SSD).  Shared with the main
+// thread through `mu`; GPU work is issued by the reader on its own streams.
+constexpr int kMaxDepth = 16;  // tile ring slots (pinned-host and SSD)
+struct SsdJob {
+  int block = -1;
+  std::vector<cudaEvent_t> wait;  // host-waited before the block's states are read
+};
+struct SsdTile {
+  int slot = 0, fd = -1;
+  uint64_t foff = 0, stride = 0, bytes = 0;
+};
+struct SsdEngine {
+  std::thread reader, writer;
+  std::mutex mu;
+  std::condition_variable cv;
+  std::deque<SsdJob> jobs;
+  std::deque<SsdTile> wq;
+  int slot_busy[kMaxDepth] = {};  // a tile in this slot still awaits its write-back
+  bool stop = false;
+  uint64_t jobs_in = 0, jobs_out = 0, tiles_in = 0, tiles_out = 0;
+  int err = 0;
+  std::string msg;
+  float* h_ring = nullptr;  // pinned: depth x {theta, m, v} x tile
+  float* d_ring = nullptr;  // device: the same shape
+  cudaStream_t s_in = nullptr, s_k = nullptr, s_out = nullptr;
+  cudaEvent_t ev_h2d[kMaxDepth] = {}, ev_d2h[kMaxDepth] = {}, ev_k1[kMaxDepth] = {};
+  uint64_t ring_k = 0;
+  double read_s = 0, write_s = 0;  // host seconds inside pread / pwrite
+  uint64_t read_bytes = 0, write_bytes = 0;
 };
 
 // One host-handler invocation (owned by the callback, deleted when done).
@@ -98,7 +145,7 @@ struct TimingPair {
 
 struct Ctx {
   bool inited = false;
-  int sticky = 0;
+  std::atomic<int> sticky{0};
   char sticky_msg[1024] = "";
   int device = 0, rank = 0, world = 1;
   ratel_config cfg{};
@@ -109,7 +156,7 @@ struct Ctx {
   // s_opt joins each (ev_done) so it stays ordered after every grad read.
   cudaStream_t s_k[2] = {nullptr, nullptr};
   unsigned k_next = 0;
-  static constexpr int kNS = 8;  // every stream, for the sync cross-waits
+  static constexpr int kNS = 11;  // every stream (8 + the SSD engine's 3), for the sync cross-waits
   cudaEvent_t ev_end[kNS] = {};
   cudaEvent_t ev_norm = nullptr;  // clip: global norm final (on s_opt)
   double* h_sumsq = nullptr;      // clip + HOST_COMPUTE: pinned copy of the norm
@@ -130,7 +177,7 @@ struct Ctx {
   // (s_k[0], s_k[1], s_tile, s_opt): launches on one stream are serialised,
   // so each counter's value at a launch is known on the host (ctr_base).
   unsigned long long* d_ctr = nullptr;
-  unsigned long long ctr_base[4] = {0, 0, 0, 0};
+  unsigned long long ctr_base[5] = {0, 0, 0, 0, 0};  // + the SSD reader's kernel stream
   int n_peer_ranges = 0;      // ranges using the fused (peer-store) all-gather
   int n_rs_blocks = 0;        // blocks using the fused gradient reduction
   int* h_flag = nullptr;      // mapped pinned: non-finite norm seen
@@ -142,9 +189,10 @@ struct Ctx {
   // NCCL
   ncclComm_t comm = nullptr;
   // stats
-  int64_t launches = 0;
+  std::atomic<int64_t> launches{0};
   std::vector<TimingPair> tpool;
   size_t tused = 0;
+  SsdEngine* ssd = nullptr;  // created by the first RATEL_SSD registration
 };
 
 Ctx G;
@@ -182,6 +230,8 @@ int sticky_fail(int code, const char* fmt, ...) {
     if (rc_ != RATEL_OK) return rc_; \
   } while (0)
 
+std::mutex g_launch_mu;  // launch bookkeeping (timing pool, tile counters): main + SSD reader thread
+
 int entry() {
   if (!G.inited) return set_error(RATEL_ESTATE, "ratel: not initialised (call ratel_init first)");
   if (G.sticky) return set_error(G.sticky, "ratel: sticky error: %s", G.sticky_msg);
@@ -216,6 +266,7 @@ const uint16_t* grad_ptr(const ratel_range& r, const Slice& s) {
 #endif
 
 int ctr_slot(cudaStream_t st) {
+  if (G.ssd != nullptr && st == G.ssd->s_k) return 4;
   return st == G.s_k[0] ? 0 : st == G.s_k[1] ? 1 : st == G.s_tile ? 2 : 3;
 }
 
@@ -270,6 +321,7 @@ void launch_k1_rs(RsUpdateParams& Q, unsigned grid, cudaStream_t st) {
 int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* pd = nullptr,
                   const GradPeers* gp = nullptr) {
   if (nr == 0) return RATEL_OK;
+  std::lock_guard<std::mutex> lk(g_launch_mu);
   UpdateParams P{};
   uint64_t max8 = 0;
   for (int i = 0; i < nr; ++i) {
@@ -527,10 +579,293 @@ int enqueue_host_compute(Block& B) {
   return RATEL_OK;
 }
 
+// ---------------------------------------------------------------- SSD tier
+// The paper's storage pipeline (Fig. 3b): per tile, read
+// theta/m/v from the state file (reader thread, pread), H2D, the update
+// kernel, D2H, write back (writer thread, pwrite).  The reader runs ahead by
+// up to pipeline_depth tiles, so the read of tile k+1, the GPU work of tile k
+// and the write-back of tile k-1 overlap; the file sees reads and writes
+// concurrently (its queue decides the mix -- the paper's SSD is simplex and
+// orders write-back of i after read of i-1).
+constexpr uint64_t kSsdAlign = 4096;
+uint64_t ssd_stride(uint64_t len) { return (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign; }
+
+double now_s() {
+  timespec ts;
+  clock_gettime(CLOCK_MONOTONIC, &ts);
+  return ts.tv_sec + 1e-9 * ts.tv_nsec;
+}
+
+int io_full(bool rd, int fd, void* buf, uint64_t bytes, uint64_t off, std::string& msg) {
+  uint8_t* p = static_cast<uint8_t*>(buf);
+  while (bytes > 0) {
+    const ssize_t r = rd ? pread(fd, p, bytes, static_cast<off_t>(off)) : pwrite(fd, p, bytes, static_cast<off_t>(off));
+    if (r < 0 && errno == EINTR) continue;
+    if (r <= 0) {
+      msg = std::string(rd ? "pread" : "pwrite") + " of the SSD state file failed at offset " + std::to_string(off) +
+            ": " + (r < 0 ? strerror(errno) : "unexpected end of file");
+      return RATEL_EIO;
+    }
+    p += r;
+    bytes -= static_cast<uint64_t>(r);
+    off += static_cast<uint64_t>(r);
+  }
+  return RATEL_OK;
+}
+
+#define SK(call)                                                                                         \
+  do {                                                                                                   \
+    cudaError_t e_ = (call);                                                                             \
+    if (e_ != cudaSuccess) {                                                                             \
+      msg = std::string(#call) + " failed: " + cudaGetErrorString(e_);                                   \
+      return RATEL_ECUDA;                                                                                \
+    }                                                                                                    \
+  } while (0)
+
+// One block: every tile of every range of this rank's slices.
+int ssd_run_job(SsdEngine& E, const SsdJob& job, std::string& msg) {
+  for (cudaEvent_t ev : job.wait) SK(cudaEventSynchronize(ev));  // the active message: the gradient exists
+  Block& B = G.blocks[job.block];
+  const uint64_t T = G.cfg.tile_elems;
+  const int D = G.cfg.pipeline_depth;
+  bool first = true;
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const ratel_range& r = B.ranges[i];
+    const Slice& s = B.slices[i];
+    const Block::SsdRange& f = B.ssd[i];
+    const uint64_t n = s.end - s.begin;
+    for (uint64_t off = 0; off < n; off += T) {
+      const uint64_t len = std::min<uint64_t>(T, n - off);
+      const int slot = static_cast<int>(E.ring_k % static_cast<uint64_t>(D));
+      {
+        std::unique_lock<std::mutex> lk(E.mu);
+        E.cv.wait(lk, [&] { return !E.slot_busy[slot] || E.err != 0; });
+        if (E.err) return E.err;
+      }
+      float* h = E.h_ring + 3ull * slot * T;
+      float* d = E.d_ring + 3ull * slot * T;
+      const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
+      const double t0 = now_s();
+      for (int a = 0; a < 3; ++a) {
+        const int rc = io_full(true, f.fd, h + a * T, bytes, f.off + a * f.stride + off * 4, msg);
+        if (rc != RATEL_OK) return rc;
+      }
+      E.read_s += now_s() - t0;
+      E.read_bytes += 3 * bytes;
+      for (int a = 0; a < 3; ++a) SK(cudaMemcpyAsync(d + a * T, h + a * T, len * 4, cudaMemcpyHostToDevice, E.s_in));
+      SK(cudaEventRecord(E.ev_h2d[slot], E.s_in));
+      SK(cudaStreamWaitEvent(E.s_k, E.ev_h2d[slot], 0));
+      if (first) {
+        SK(cudaStreamWaitEvent(E.s_k, B.ev_grad, 0));
+        if (G.cfg.max_grad_norm > 0.0) SK(cudaStreamWaitEvent(E.s_k, G.ev_norm, 0));
+        first = false;
+      }
+      RangeDesc rd{};
+      rd.g = grad_ptr(r, s) + off;
+      rd.th = d;
+      rd.m = d + T;
+      rd.v = d + 2 * T;
+      rd.p = static_cast<uint16_t*>(r.param_bf16) + s.begin + off;
+      rd.n = len;
+      rd.wd_on = r.apply_weight_decay != 0;
+      if (launch_update(&rd, 1, E.s_k) != RATEL_OK) {
+        msg = t_err;
+        return RATEL_ECUDA;
+      }
+      SK(cudaEventRecord(E.ev_k1[slot], E.s_k));
+      SK(cudaStreamWaitEvent(E.s_out, E.ev_k1[slot], 0));
+      for (int a = 0; a < 3; ++a) SK(cudaMemcpyAsync(h + a * T, d + a * T, len * 4, cudaMemcpyDeviceToHost, E.s_out));
+      SK(cudaEventRecord(E.ev_d2h[slot], E.s_out));
+      {
+        std::lock_guard<std::mutex> lk(E.mu);
+        E.slot_busy[slot] = 1;
+        SsdTile t;
+        t.slot = slot;
+        t.fd = f.fd;
+        t.foff = f.off + off * 4;
+        t.stride = f.stride;
+        t.bytes = bytes;
+        E.wq.push_back(t);
+        ++E.tiles_in;
+      }
+      E.cv.notify_all();
+      ++E.ring_k;
+    }
+  }
+  if (first) {  // no tile on this rank: still order ev_done after the gradient
+    SK(cudaStreamWaitEvent(E.s_k, B.ev_grad, 0));
+  }
+  SK(cudaEventRecord(B.ev_done, E.s_k));
+  return RATEL_OK;
+}
+
+void ssd_fail(SsdEngine& E, int rc, const std::string& m) {
+  std::lock_guard<std::mutex> lk(E.mu);
+  if (!E.err) {
+    E.err = rc;
+    E.msg = m;
+  }
+}
+
+void ssd_reader_main(SsdEngine* E) {
+  cudaSetDevice(G.device);
+  for (;;) {
+    SsdJob job;
+    {
+      std::unique_lock<std::mutex> lk(E->mu);
+      E->cv.wait(lk, [&] { return E->stop || !E->jobs.empty(); });
+      if (E->jobs.empty()) return;  // stop
+      job = E->jobs.front();
+      E->jobs.pop_front();
+    }
+    bool failed;
+    {
+      std::lock_guard<std::mutex> lk(E->mu);
+      failed = E->err != 0;
+    }
+    if (!failed) {
+      std::string m;
+      const int rc = ssd_run_job(*E, job, m);
+      if (rc != RATEL_OK) ssd_fail(*E, rc, "SSD reader: " + m);
+    }
+    {
+      std::lock_guard<std::mutex> lk(E->mu);
+      ++E->jobs_out;
+    }
+    E->cv.notify_all();
+  }
+}
+
+void ssd_writer_main(SsdEngine* E) {
+  cudaSetDevice(G.device);
+  const uint64_t T = G.cfg.tile_elems;
+  for (;;) {
+    SsdTile t;
+    bool failed;
+    {
+      std::unique_lock<std::mutex> lk(E->mu);
+      E->cv.wait(lk, [&] { return E->stop || !E->wq.empty(); });
+      if (E->wq.empty()) return;  // stop
+      t = E->wq.front();
+      E->wq.pop_front();
+      failed = E->err != 0;
+    }
+    if (!failed) {
+      std::string m;
+      int rc = RATEL_OK;
+      const cudaError_t e = cudaEventSynchronize(E->ev_d2h[t.slot]);  // the tile's states are back in the slot
+      if (e != cudaSuccess) {
+        rc = RATEL_ECUDA;
+        m = std::string("cudaEventSynchronize(d2h) failed: ") + cudaGetErrorString(e);
+      }
+      const float* h = E->h_ring + 3ull * t.slot * T;
+      const double t0 = now_s();
+      for (int a = 0; a < 3 && rc == RATEL_OK; ++a)
+        rc = io_full(false, t.fd, const_cast<float*>(h + a * T), t.bytes, t.foff + a * t.stride, m);
+      E->write_s += now_s() - t0;
+      E->write_bytes += 3 * t.bytes;
+      if (rc != RATEL_OK) ssd_fail(*E, rc, "SSD writer: " + m);
+    }
+    {
+      std::lock_guard<std::mutex> lk(E->mu);
+      E->slot_busy[t.slot] = 0;
+      ++E->tiles_out;
+    }
+    E->cv.notify_all();
+  }
+}
+
+int ssd_create() {
+  SsdEngine* E = new SsdEngine();
+  G.ssd = E;  // destroy_all() tears down whatever was created
+  const size_t n = static_cast<size_t>(G.cfg.pipeline_depth) * 3 * G.cfg.tile_elems;
+  CK(cudaHostAlloc(&E->h_ring, n * sizeof(float), cudaHostAllocDefault));
+  CK(cudaMalloc(&E->d_ring, n * sizeof(float)));
+  int least = 0, greatest = 0;
+  CK(cudaDeviceGetStreamPriorityRange(&least, &greatest));
+  CK(cudaStreamCreateWithPriority(&E->s_in, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&E->s_k, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&E->s_out, cudaStreamNonBlocking, greatest));
+  for (int k = 0; k < kMaxDepth; ++k) {
+    CK(cudaEventCreateWithFlags(&E->ev_h2d[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&E->ev_k1[k], cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&E->ev_d2h[k], cudaEventDisableTiming | cudaEventBlockingSync));
+  }
+  E->reader = std::thread(ssd_reader_main, E);
+  E->writer = std::thread(ssd_writer_main, E);
+  return RATEL_OK;
+}
+
+void ssd_destroy() {
+  SsdEngine* E = G.ssd;
+  if (E == nullptr) return;
+  {
+    std::lock_guard<std::mutex> lk(E->mu);
+    E->stop = true;
+  }
+  E->cv.notify_all();
+  if (E->reader.joinable()) E->reader.join();
+  if (E->writer.joinable()) E->writer.join();
+  for (cudaStream_t s : {E->s_in, E->s_k, E->s_out})
+    if (s) cudaStreamSynchronize(s);
+  for (int k = 0; k < kMaxDepth; ++k) {
+    if (E->ev_h2d[k]) cudaEventDestroy(E->ev_h2d[k]);
+    if (E->ev_k1[k]) cudaEventDestroy(E->ev_k1[k]);
+    if (E->ev_d2h[k]) cudaEventDestroy(E->ev_d2h[k]);
+  }
+  for (cudaStream_t s : {E->s_in, E->s_k, E->s_out})
+    if (s) cudaStreamDestroy(s);
+  if (E->h_ring) cudaFreeHost(E->h_ring);
+  if (E->d_ring) cudaFree(E->d_ring);
+  delete E;
+  G.ssd = nullptr;
+}
+
+// Hand block B to the reader (hand-off / arm time).  `wait`: events the
+// reader host-waits before touching B's states.
+int ssd_submit(Block& B, int id, std::vector<cudaEvent_t> wait) {
+  SsdEngine& E = *G.ssd;
+  {
+    std::lock_guard<std::mutex> lk(E.mu);
+    SsdJob j;
+    j.block = id;
+    j.wait = std::move(wait);
+    E.jobs.push_back(std::move(j));
+    B.ssd_seq = ++E.jobs_in;
+  }
+  E.cv.notify_all();
+  return RATEL_OK;
+}
+
+// Wait until the reader issued every submitted job (and, if `writes`, the
+// writer finished every write-back); report an engine failure as sticky.
+int ssd_drain(bool writes, uint64_t upto_job = 0) {
+  if (G.ssd == nullptr) return RATEL_OK;
+  SsdEngine& E = *G.ssd;
+  std::unique_lock<std::mutex> lk(E.mu);
+  const uint64_t want = upto_job ? upto_job : E.jobs_in;
+  E.cv.wait(lk, [&] { return E.err != 0 || (E.jobs_out >= want && (!writes || E.tiles_out == E.tiles_in)); });
+  if (E.err) {
+    // let the threads finish draining their queues before reporting
+    E.cv.wait(lk, [&] { return E.jobs_out == E.jobs_in && E.tiles_out == E.tiles_in; });
+    const std::string m = E.msg;
+    const int rc = E.err;
+    lk.unlock();
+    return sticky_fail(rc, "%s", m.c_str());
+  }
+  return RATEL_OK;
+}
+
 // Enqueue the handler of block B (its s_opt wait on ev_grad was issued at
 // hand-off).  Device residency: one K1 launch over the rank's slices of all
 // ranges.  Pinned-host: the tile ring.
-int enqueue_block(Block& B) {
+int enqueue_block(Block& B, const std::vector<cudaEvent_t>* ssd_wait = nullptr) {
+  if (B.residency == RATEL_SSD) {
+    const int id = static_cast<int>(&B - G.blocks.data());
+    RK(ssd_submit(B, id, ssd_wait ? *ssd_wait : std::vector<cudaEvent_t>{B.ev_grad}));
+    B.enqueued = true;
+    return RATEL_OK;
+  }
   cudaStream_t ks = G.s_opt;
   if (B.residency == RATEL_DEVICE) {
     // Alternate update streams: this block's kernel can take the SMs the
@@ -657,6 +992,7 @@ void reset_step_state() {
 }
 
 void destroy_all() {
+  ssd_destroy();  // joins the SSD threads before their streams and buffers go
   for (int id : G.reg) {
     Block& B = G.blocks[id];
     if (B.ev_grad) cudaEventDestroy(B.ev_grad);
@@ -740,8 +1076,8 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK((prepare_k1<RATEL_ADAM_L2, true>()));
   if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
   G.k2_grid = G.sms * 4;
-  CK(cudaMalloc(&G.d_ctr, 4 * sizeof(unsigned long long)));
-  CK(cudaMemset(G.d_ctr, 0, 4 * sizeof(unsigned long long)));
+  CK(cudaMalloc(&G.d_ctr, 5 * sizeof(unsigned long long)));
+  CK(cudaMemset(G.d_ctr, 0, 5 * sizeof(unsigned long long)));
   CK(cudaMalloc(&G.d_sumsq, 3 * sizeof(double)));
   CK(cudaMemset(G.d_sumsq, 0, 3 * sizeof(double)));
   G.d_barrier = G.d_sumsq + 2;
@@ -848,8 +1184,15 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     return set_error(RATEL_EINVAL, "ratel_register_block: block %d already registered", block_id);
   if (ranges == nullptr || n_ranges < 1 || n_ranges > RATEL_MAX_RANGES_PER_BLOCK)
     return set_error(RATEL_EINVAL, "ratel_register_block: need 1..%d ranges", RATEL_MAX_RANGES_PER_BLOCK);
-  if (residency != RATEL_DEVICE && residency != RATEL_PINNED_HOST && residency != RATEL_HOST_COMPUTE)
+  if (residency != RATEL_DEVICE && residency != RATEL_PINNED_HOST && residency != RATEL_HOST_COMPUTE &&
+      residency != RATEL_SSD)
     return set_error(RATEL_EINVAL, "ratel_register_block: bad residency %d", residency);
+  if (residency == RATEL_SSD) {
+    if (G.comm != nullptr)
+      return set_error(RATEL_EINVAL, "ratel_register_block: RATEL_SSD blocks need a single rank without NCCL");
+    if (G.cfg.tile_elems % 1024u)
+      return set_error(RATEL_EINVAL, "ratel_register_block: RATEL_SSD needs cfg.tile_elems to be a multiple of 1024");
+  }
   std::vector<Slice> slices(n_ranges);
   for (int i = 0; i < n_ranges; ++i) {
     const ratel_range& r = ranges[i];
@@ -858,14 +1201,15 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     const bool has = slices[i].end > slices[i].begin;
     if (r.param_bf16 == nullptr || r.grad_bf16 == nullptr)
       return set_error(RATEL_EINVAL, "range %d: param/grad pointer is NULL", i);
-    if (has && (r.master == nullptr || r.exp_avg == nullptr || r.exp_avg_sq == nullptr))
+    const bool states = residency != RATEL_SSD;  // SSD: the states are in the file (ratel_register_ssd)
+    if (states && has && (r.master == nullptr || r.exp_avg == nullptr || r.exp_avg_sq == nullptr))
       return set_error(RATEL_EINVAL, "range %d: state pointer is NULL", i);
     const void* ps[5] = {r.param_bf16, r.grad_bf16, r.master, r.exp_avg, r.exp_avg_sq};
     for (const void* p : ps)
       if (p && !aligned16(p)) return set_error(RATEL_EINVAL, "range %d: pointers must be 16-byte aligned", i);
     RK(check_ptr(r.param_bf16, true, "param_bf16", i));
     RK(check_ptr(r.grad_bf16, true, "grad_bf16", i));
-    if (has) {
+    if (states && has) {
       const bool dev = residency == RATEL_DEVICE;  // PINNED_HOST and HOST_COMPUTE: page-locked host
       RK(check_ptr(r.master, dev, "master", i));
       RK(check_ptr(r.exp_avg, dev, "exp_avg", i));
@@ -905,7 +1249,12 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     }
     CK(cudaEventCreateWithFlags(&B.ev_gh, cudaEventDisableTiming));
   }
-  CK(cudaEventCreateWithFlags(&B.ev_grad, cudaEventDisableTiming));
+  if (residency == RATEL_SSD) {
+    if (G.ssd == nullptr) RK(ssd_create());
+    B.ssd.assign(n_ranges, Block::SsdRange());
+  }
+  // (blocking sync: the SSD reader thread sleeps on ev_grad instead of spinning)
+  CK(cudaEventCreateWithFlags(&B.ev_grad, cudaEventDisableTiming | cudaEventBlockingSync));
   CK(cudaEventCreateWithFlags(&B.ev_done, cudaEventDisableTiming));
   B.ranges.assign(ranges, ranges + n_ranges);
   B.slices = slices;
@@ -924,8 +1273,8 @@ int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_pa
   Block& B = G.blocks[block_id];
   if (range_idx < 0 || range_idx >= static_cast<int>(B.ranges.size()))
     return set_error(RATEL_EINVAL, "ratel_register_peer_params: range %d out of range", range_idx);
-  if (B.residency == RATEL_HOST_COMPUTE)
-    return set_error(RATEL_EINVAL, "ratel_register_peer_params: HOST_COMPUTE blocks use the NCCL all-gather");
+  if (B.residency == RATEL_HOST_COMPUTE || B.residency == RATEL_SSD)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_params: not for HOST_COMPUTE / SSD blocks");
   if (peer_params == nullptr || n != G.world || G.world - 1 > kMaxPeers)
     return set_error(RATEL_EINVAL, "ratel_register_peer_params: need world_size (%d <= %d) pointers", G.world,
                      kMaxPeers + 1);
@@ -951,8 +1300,8 @@ int ratel_register_peer_grads(int block_id, int range_idx, const void* const* ra
   Block& B = G.blocks[block_id];
   if (range_idx < 0 || range_idx >= static_cast<int>(B.ranges.size()))
     return set_error(RATEL_EINVAL, "ratel_register_peer_grads: range %d out of range", range_idx);
-  if (B.residency == RATEL_HOST_COMPUTE)
-    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: not for HOST_COMPUTE blocks");
+  if (B.residency == RATEL_HOST_COMPUTE || B.residency == RATEL_SSD)
+    return set_error(RATEL_EINVAL, "ratel_register_peer_grads: not for HOST_COMPUTE / SSD blocks");
   if (B.ranges[range_idx].grad_is_rank_slice)
     return set_error(RATEL_EINVAL, "ratel_register_peer_grads: the range's grad must be full-range (grad_is_rank_slice = 0)");
   if (rank_grads == nullptr || n != G.world || G.world > kMaxRanks)
@@ -980,6 +1329,37 @@ int ratel_register_peer_grads(int block_id, int range_idx, const void* const* ra
   if (!B.rs) ++G.n_rs_blocks;
   B.rs = true;
   return RATEL_OK;
+}
+
+int ratel_register_ssd(int block_id, int range_idx, int fd, uint64_t offset) {
+  RK(entry());
+  if (G.armed || G.n_handed > 0) return set_error(RATEL_ESTATE, "ratel_register_ssd: a step is in flight");
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
+    return set_error(RATEL_EINVAL, "ratel_register_ssd: block %d is not registered", block_id);
+  Block& B = G.blocks[block_id];
+  if (B.residency != RATEL_SSD) return set_error(RATEL_EINVAL, "ratel_register_ssd: block %d is not RATEL_SSD", block_id);
+  if (range_idx < 0 || range_idx >= static_cast<int>(B.ranges.size()))
+    return set_error(RATEL_EINVAL, "ratel_register_ssd: range %d out of range", range_idx);
+  if (offset % kSsdAlign) return set_error(RATEL_EINVAL, "ratel_register_ssd: offset must be a multiple of 4096");
+  struct stat st{};
+  if (fd < 0 || fstat(fd, &st) != 0) return set_error(RATEL_EINVAL, "ratel_register_ssd: fd %d is not open", fd);
+  const int fl = fcntl(fd, F_GETFL);
+  if (fl < 0 || (fl & O_ACCMODE) != O_RDWR) return set_error(RATEL_EINVAL, "ratel_register_ssd: fd must be open O_RDWR");
+  const Slice& s = B.slices[range_idx];
+  const uint64_t stride = ssd_stride(s.end - s.begin);
+  if (static_cast<uint64_t>(st.st_size) < offset + 3 * stride)
+    return set_error(RATEL_EINVAL, "ratel_register_ssd: the file holds %lld bytes, needs %llu", (long long)st.st_size,
+                     static_cast<unsigned long long>(offset + 3 * stride));
+  B.ssd[range_idx].fd = fd;
+  B.ssd[range_idx].off = offset;
+  B.ssd[range_idx].stride = stride;
+  return RATEL_OK;
+}
+
+uint64_t ratel_ssd_range_bytes(uint64_t numel, int world_size, int rank) {
+  if (world_size < 1 || rank < 0 || rank >= world_size) return 0;
+  const Slice s = slice_of(numel, world_size, rank);
+  return 3 * ssd_stride(s.end - s.begin);
 }
 
 int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay, int64_t step) {
@@ -1026,7 +1406,9 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
   if (!G.pending.empty())
     for (cudaStream_t st : {G.s_h2d, G.s_d2h, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
       for (int id : G.pending) CK(cudaStreamWaitEvent(st, G.blocks[id].ev_grad, 0));
-  for (int id : G.pending) RK(enqueue_block(G.blocks[id]));
+  std::vector<cudaEvent_t> all_grads;  // SSD: no state is read before the whole backward
+  for (int id : G.pending) all_grads.push_back(G.blocks[id].ev_grad);
+  for (int id : G.pending) RK(enqueue_block(G.blocks[id], &all_grads));
   G.pending.clear();
   return RATEL_OK;
 }
@@ -1039,6 +1421,10 @@ int ratel_offload_grad_chunk(int block_id, void* stream) {
   Block& B = G.blocks[block_id];
   if (B.handed_off)
     return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d already handed off this step", block_id);
+  if (B.residency == RATEL_SSD)
+    for (size_t i = 0; i < B.ssd.size(); ++i)
+      if (B.ssd[i].fd < 0 && B.slices[i].end > B.slices[i].begin)
+        return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d range %zu has no SSD file", block_id, i);
   CK(cudaEventRecord(B.ev_grad, static_cast<cudaStream_t>(stream)));
   CK(cudaStreamWaitEvent(G.s_opt, B.ev_grad, 0));
   if (B.rs && G.comm != nullptr) {
@@ -1071,6 +1457,7 @@ int ratel_block_wait(int block_id, void* stream) {
   const Block& B = G.blocks[block_id];
   if (B.handed_off && !B.enqueued)
     return set_error(RATEL_ESTATE, "ratel_block_wait: block %d's update is not enqueued yet", block_id);
+  if (B.residency == RATEL_SSD && B.enqueued) RK(ssd_drain(false, B.ssd_seq));  // its ev_done is recorded
   if (B.rs && G.comm != nullptr && B.enqueued) {
     // Peers read this rank's G16 too: release it only after every rank's
     // update of the block (collective: every rank calls block_wait alike).
@@ -1104,8 +1491,12 @@ int ratel_sync(void* stream) {
     CK(cudaStreamWaitEvent(G.s_comm, G.ev_end[5], 0));
     NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
   }
-  constexpr int NS = Ctx::kNS;
-  cudaStream_t ss[NS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]};
+  // SSD: every job issued to the GPU and every state write-back in the file
+  RK(ssd_drain(true));
+  const int NS = G.ssd != nullptr ? Ctx::kNS : Ctx::kNS - 3;
+  cudaStream_t ss[Ctx::kNS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1],
+                               G.ssd ? G.ssd->s_in : nullptr, G.ssd ? G.ssd->s_k : nullptr,
+                               G.ssd ? G.ssd->s_out : nullptr};
   for (int i = 0; i < NS; ++i) CK(cudaEventRecord(G.ev_end[i], ss[i]));
   // Order the internal streams too: the next step's stage-in must not read
   // host states still being written back, and its K1 must not overwrite a

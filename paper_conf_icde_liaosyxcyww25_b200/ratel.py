@@ -23,10 +23,12 @@ RATEL_ECUDA = -3
 RATEL_ENCCL = -4
 RATEL_ENOMEM = -5
 RATEL_ENONFINITE = -6
+RATEL_EIO = -7
 
 RATEL_DEVICE = 0
 RATEL_PINNED_HOST = 1
 RATEL_HOST_COMPUTE = 2
+RATEL_SSD = 3
 RATEL_ADAMW = 0
 RATEL_ADAM_L2 = 1
 RATEL_STAGING_PIPELINED = 0
@@ -38,7 +40,8 @@ RATEL_MAX_BLOCKS = 4096
 RATEL_MAX_RANGES_PER_BLOCK = 32
 
 _NAMES = {0: "RATEL_OK", -1: "RATEL_EINVAL", -2: "RATEL_ESTATE", -3: "RATEL_ECUDA",
-          -4: "RATEL_ENCCL", -5: "RATEL_ENOMEM", -6: "RATEL_ENONFINITE"}
+          -4: "RATEL_ENCCL", -5: "RATEL_ENOMEM", -6: "RATEL_ENONFINITE",
+          -7: "RATEL_EIO"}
 
 
 class RatelError(RuntimeError):
@@ -94,6 +97,8 @@ def load_library(path: str = _LIB_PATH, strict: bool = True):
         "ratel_block_wait": (I, [I, P]),
         "ratel_register_peer_params": (I, [I, I, ctypes.POINTER(P), I]),
         "ratel_register_peer_grads": (I, [I, I, ctypes.POINTER(P), I, D]),
+        "ratel_register_ssd": (I, [I, I, I, U64]),
+        "ratel_ssd_range_bytes": (U64, [U64, I, I]),
         "ratel_finalize": (I, []),
         "ratel_last_error": (ctypes.c_char_p, []),
         "ratel_padded_numel": (U64, [U64, I]),
@@ -182,6 +187,16 @@ def ratel_register_peer_grads(block_id: int, range_idx: int, rank_grads, grad_sc
     ptrs = [(p.data_ptr() if hasattr(p, "data_ptr") else (int(p) if p else None)) for p in rank_grads]
     arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
     _check(_lib.ratel_register_peer_grads(block_id, range_idx, arr, len(ptrs), grad_scale))
+
+
+def ratel_register_ssd(block_id: int, range_idx: int, fd: int, offset: int) -> None:
+    """RATEL_SSD block: the range's theta/m/v live in file `fd` at `offset`
+    (layout: ratel_ssd_range_bytes)."""
+    _check(_lib.ratel_register_ssd(block_id, range_idx, fd, offset))
+
+
+def ratel_ssd_range_bytes(numel: int, world_size: int = 1, rank: int = 0) -> int:
+    return int(_lib.ratel_ssd_range_bytes(numel, world_size, rank))
 
 
 def ratel_adam_step(lr: float, beta1: float, beta2: float, eps: float, weight_decay: float, step: int) -> None:

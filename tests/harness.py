@@ -95,3 +95,55 @@ class GpuBlock:
         n = self.sizes[i]
         return dict(p32=self.master[i][:n].cpu().numpy(), m32=self.m[i][:n].cpu().numpy(),
                     v32=self.v[i][:n].cpu().numpy(), p16=torch_to_u16(self.p16[i][:n]))
+
+
+class SsdBlock(GpuBlock):
+    """A RATEL_SSD block: P16 and grads on the device, theta/m/v in a state
+    file (layout of ratel_ssd_range_bytes; the test writes theta0 and zeros
+    through a buffered fd, the library gets an O_DIRECT fd)."""
+
+    def __init__(self, block_id: int, sizes, device, path, wd_flags=None, direct: bool = True, base: int = 0):
+        super().__init__(block_id, sizes, device, wd_flags=wd_flags)
+        import os
+        self.path = str(path)
+        self.offs_file = []
+        off = base
+        for n in self.sizes:
+            self.offs_file.append(off)
+            off += R.ratel_ssd_range_bytes(n, 1, 0)
+        self.file_bytes = off
+        self.strides = [R.ratel_ssd_range_bytes(n, 1, 0) // 3 for n in self.sizes]
+        fdw = os.open(self.path, os.O_RDWR | os.O_CREAT, 0o600)
+        os.ftruncate(fdw, max(os.fstat(fdw).st_size, off))
+        for i, n in enumerate(self.sizes):
+            th = self.master[i][:n].cpu().numpy()
+            os.pwrite(fdw, th.tobytes(), self.offs_file[i])
+            z = np.zeros(n, np.float32).tobytes()
+            os.pwrite(fdw, z, self.offs_file[i] + self.strides[i])
+            os.pwrite(fdw, z, self.offs_file[i] + 2 * self.strides[i])
+        os.fsync(fdw)
+        self.fd_check = fdw
+        self.fd = os.open(self.path, os.O_RDWR | (os.O_DIRECT if direct else 0))
+        # the device states of the base class are not used
+        self.master = self.m = self.v = None
+
+    def ranges(self):
+        return [R.make_range(self.p16[i], self.g16[i], None, None, None, n, self.wd[i])
+                for i, n in enumerate(self.sizes)]
+
+    def register(self):
+        R.ratel_register_block(self.id, self.ranges(), R.RATEL_SSD)
+        for i in range(len(self.sizes)):
+            R.ratel_register_ssd(self.id, i, self.fd, self.offs_file[i])
+
+    def gpu_state(self, i: int) -> dict:
+        import os
+        n = self.sizes[i]
+        rd = lambda k: np.frombuffer(os.pread(self.fd_check, 4 * n, self.offs_file[i] + k * self.strides[i]),
+                                     dtype=np.float32).copy()
+        return dict(p32=rd(0), m32=rd(1), v32=rd(2), p16=torch_to_u16(self.p16[i][:n]))
+
+    def close(self):
+        import os
+        os.close(self.fd)
+        os.close(self.fd_check)

@@ -124,3 +124,12 @@ def test_struct_layouts_match_header():
     # ratel_range: 2 ptrs, int, 3 ptrs, uint64, int -> 64 bytes
     assert ctypes.sizeof(R.ratel_range) == 64
     assert R.ratel_range.master.offset == 24 and R.ratel_range.numel.offset == 48
+
+
+def test_ssd_range_bytes():
+    """3 fp32 arrays of the rank slice, each padded to 4096 bytes (pure host)."""
+    for n, world, rank in [(1, 1, 0), (1024, 1, 0), (1025, 1, 0), (300_001, 1, 0), (300_001, 4, 3), (16, 4, 3)]:
+        b, e = R.ratel_rank_slice(n, world, rank)
+        want = 3 * ((4 * (e - b) + 4095) // 4096 * 4096)
+        assert R.ratel_ssd_range_bytes(n, world, rank) == want
+    assert R.ratel_ssd_range_bytes(10, 0, 0) == 0
