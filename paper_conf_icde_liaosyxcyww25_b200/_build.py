@@ -15,8 +15,8 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libratel.so")
-SOURCES = ["ratel_runtime.cu", "ratel_gen.cu", "ratel_host_adam.cpp"]
-HEADERS = ["ratel_kernels.cuh", "ratel_bf16.cuh", "nccl_dl.h", "ratel_host_adam.h"]
+SOURCES = ["ratel_runtime.cu", "ratel_gen.cu", "ratel_host_adam.cpp", "ratel_plan.cpp"]
+HEADERS = ["ratel_kernels.cuh", "ratel_bf16.cuh", "nccl_dl.h", "ratel_host_adam.h", "ratel_plan_impl.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

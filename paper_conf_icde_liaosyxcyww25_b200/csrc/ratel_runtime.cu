@@ -38,6 +38,7 @@
 #include "nccl_dl.h"
 #include "ratel.h"
 #include "ratel_host_adam.h"
+#include "ratel_plan_impl.h"
 #include "ratel_kernels.cuh"
 
 namespace {
@@ -1102,6 +1103,10 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
 }
 
 }  // namespace
+
+// Host-only parts of the library (the swap planner) report through the same
+// thread-local message as the runtime.
+int ratel::report_error(int code, const char* msg) { return set_error(code, "%s", msg); }
 
 extern "C" {
 

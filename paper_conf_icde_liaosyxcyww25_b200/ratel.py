@@ -78,6 +78,21 @@ class ratel_range(ctypes.Structure):
     ]
 
 
+class ratel_swap_model(ctypes.Structure):
+    """include/ratel_plan.h: Table I quantities."""
+    _fields_ = [(f, ctypes.c_double) for f in
+                ("thp_g", "bw_g", "bw_s2m", "bw_m2s", "mem_m_avail", "params", "flop_f")]
+
+
+class ratel_swap_layer(ctypes.Structure):
+    _fields_ = [("act_bytes", ctypes.c_double), ("recompute_flop", ctypes.c_double)]
+
+
+class ratel_swap_plan(ctypes.Structure):
+    _fields_ = [("n_swap", ctypes.c_int)] + [(f, ctypes.c_double) for f in
+                                              ("a_g2m", "flop_r", "t_f", "t_b", "t_iter", "t_min")]
+
+
 def load_library(path: str = _LIB_PATH, strict: bool = True):
     """Load a libratel.so build and declare its signatures (tools load
     build-variant copies through this; the package uses the in-tree one)."""
@@ -114,6 +129,11 @@ def load_library(path: str = _LIB_PATH, strict: bool = True):
         "ratel_gen_grad16": (I, [P, U64, U64, U64, P]),
         "ratel_test_bf16_rne": (I, [P, P, U64, P]),
         "ratel_test_fill_f32": (I, [P, U64, ctypes.c_float, P]),
+        "ratel_swap_iter_time": (I, [ctypes.POINTER(ratel_swap_model), D, D, ctypes.POINTER(D),
+                                     ctypes.POINTER(D)]),
+        "ratel_swap_recompute_flop": (I, [ctypes.POINTER(ratel_swap_layer), I, D, D, ctypes.POINTER(D)]),
+        "ratel_plan_activation_swap": (I, [ctypes.POINTER(ratel_swap_layer), I, ctypes.POINTER(ratel_swap_model),
+                                           D, ctypes.POINTER(I), ctypes.POINTER(ratel_swap_plan)]),
     }
     for name, (res, args) in sig.items():
         if not strict and not hasattr(lib, name):
@@ -197,6 +217,42 @@ def ratel_register_ssd(block_id: int, range_idx: int, fd: int, offset: int) -> N
 
 def ratel_ssd_range_bytes(numel: int, world_size: int = 1, rank: int = 0) -> int:
     return int(_lib.ratel_ssd_range_bytes(numel, world_size, rank))
+
+
+# ---------------------------------------------------------------- swap planner
+# include/ratel_plan.h (§IV-D, Eq. 1-8, Algorithm 1): host-only.
+def _swap_layers(layers):
+    """layers: iterable of (act_bytes, recompute_flop) pairs."""
+    layers = list(layers)
+    arr = (ratel_swap_layer * max(len(layers), 1))()
+    for i, (a, f) in enumerate(layers):
+        arr[i].act_bytes, arr[i].recompute_flop = float(a), float(f)
+    return arr, len(layers)
+
+
+def ratel_swap_iter_time(model: ratel_swap_model, a_g2m: float, flop_r: float):
+    """Eq. 4 / Eq. 5 -> (T_f, T_b) in seconds."""
+    tf, tb = ctypes.c_double(), ctypes.c_double()
+    _check(_lib.ratel_swap_iter_time(ctypes.byref(model), a_g2m, flop_r, ctypes.byref(tf), ctypes.byref(tb)))
+    return tf.value, tb.value
+
+
+def ratel_swap_recompute_flop(layers, flop_f: float, a_g2m: float) -> float:
+    """Eq. 7: FLOP_r after swapping a_g2m bytes along the OB order."""
+    arr, n = _swap_layers(layers)
+    out = ctypes.c_double()
+    _check(_lib.ratel_swap_recompute_flop(arr, n, flop_f, a_g2m, ctypes.byref(out)))
+    return out.value
+
+
+def ratel_plan_activation_swap(layers, model: ratel_swap_model, a_inter_block: float):
+    """Algorithm 1 -> (swapped layer indices in OB order, full OB order, plan)."""
+    arr, n = _swap_layers(layers)
+    order = (ctypes.c_int * max(n, 1))()
+    plan = ratel_swap_plan()
+    _check(_lib.ratel_plan_activation_swap(arr, n, ctypes.byref(model), a_inter_block, order, ctypes.byref(plan)))
+    full = list(order)[:n]
+    return full[:plan.n_swap], full, plan
 
 
 def ratel_adam_step(lr: float, beta1: float, beta2: float, eps: float, weight_decay: float, step: int) -> None:

@@ -16,7 +16,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 def declared_functions():
     names = []
-    for h in ("ratel.h", "ratel_gen.h"):
+    for h in ("ratel.h", "ratel_gen.h", "ratel_plan.h"):
         src = open(os.path.join(ROOT, "include", h)).read()
         src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
         names += re.findall(r"^[A-Za-z_][\w\s\*]*?\b(ratel_\w+)\s*\(", src, flags=re.M)
