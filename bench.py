@@ -324,8 +324,10 @@ class SynthBackward:
         self.vocab_rows = vocab_rows
         self.dYv = mk(2048, vocab_rows) if vocab_rows else None
 
-    def block(self, b, slot):
-        """GEMMs of block b; dW into ring slot `slot` (flat, same layout as P16)."""
+    def block(self, b, slot, on_linear=None):
+        """GEMMs of block b; dW into ring slot `slot` (flat, same layout as P16).
+        The linears run in backward order (fc2, fc1, proj, qkv); on_linear(j)
+        is called after linear j's dW (per-tensor hand-off)."""
         import torch
         h, T = self.h, self.T
         P = self.p16[b]
@@ -341,14 +343,19 @@ class SynthBackward:
                 t1 = min(T, t0 + 2048)
                 out.addmm_(self.dYv[:t1 - t0].t(), X[t0:t1])
             return
-        off = 0
+        offs, off = [], 0
         for (o, i) in linears(h):
+            offs.append(off)
+            off += o * i
+        for j in reversed(range(len(offs))):
+            (o, i), off = linears(h)[j], offs[j]
             W = P[off:off + o * i].view(o, i)
             X = self.X[i // h]
             dY = self.dY[o // h]
             torch.mm(dY, W, out=self.dX[:, :i])                          # dX = dY W
             torch.mm(dY.t(), X, out=G[off:off + o * i].view(o, i))         # dW = dY^T X
-            off += o * i
+            if on_linear is not None:
+                on_linear(j)
 
 
 SIM_COMM_NONE = False   # --sim-comm-none: N ranks on ONE GPU, gloo group, no NCCL (test mode)

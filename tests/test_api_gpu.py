@@ -107,3 +107,36 @@ def test_paper_api_state_dict_resume(cuda_dev):
     for a, b in zip(want, got):
         assert torch.equal(a.view(torch.int16) if a.dtype == torch.bfloat16 else a.view(torch.int32),
                            b.view(torch.int16) if b.dtype == torch.bfloat16 else b.view(torch.int32))
+
+
+@pytest.mark.parametrize("residency", ["device", "host"])
+def test_paper_api_tensor_granularity_bitwise(cuda_dev, residency):
+    """granularity="tensor" (one unit per weight matrix + one for the block's
+    biases/norms, each handed off by its own hook as soon as its gradient is
+    complete) updates every element exactly as block granularity does (R16):
+    the model's bf16 parameters and fp32 masters agree bitwise after 4 steps,
+    and every unit was handed off during backward."""
+    def build():
+        torch.manual_seed(2)
+        return torch.nn.Sequential(*[Block(64) for _ in range(3)]).to(cuda_dev)
+
+    x = torch.randn(48, 64, device=cuda_dev, dtype=torch.bfloat16)
+    out = {}
+    for gran in ("block", "tensor"):
+        with Ratel_init():
+            model = build()
+            opt = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in model], residency=residency,
+                                             granularity=gran))
+            assert len(opt.block_ids) == (3 if gran == "block" else 3 * 3)   # fc1.w, fc2.w, {biases, ln}
+            for _ in range(4):
+                opt.begin_step()
+                model(x).float().pow(2).mean().backward()
+                assert len(opt._handed) == len(opt.block_ids)   # all units by hooks, during backward
+                opt.end_step()
+            torch.cuda.synchronize()
+            out[gran] = ([p.detach().view(torch.int16).cpu().clone() for p in model.parameters()],
+                         sorted(torch.cat([r.master.cpu() for rs in opt.blocks for r in rs]).view(torch.int32).tolist()))
+            opt.remove_hooks()
+    for a, b in zip(out["block"][0], out["tensor"][0]):
+        assert torch.equal(a, b)
+    assert out["block"][1] == out["tensor"][1]

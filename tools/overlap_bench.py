@@ -54,6 +54,34 @@ def run(args):
     vocab = bench.VOCAB if len(sizes) == L + 1 else 0
     hi = torch.cuda.Stream(priority=-2)
     order = list(reversed(range(len(sizes))))
+    # --granularity tensor: every linear of a block (its weights; the last one
+    # also carries the block's 13h biases/LN) is its own registered unit,
+    # handed off right after its dW GEMM -- the paper's per-tensor hand-off
+    # (P:L1038-1041).  Unit id = b*K + j, j = linear index (qkv 0 .. fc2 3).
+    K = 4 if args.granularity == "tensor" else 1
+    units = {}            # block -> [ratel_range per unit]
+    for b, n in enumerate(sizes):
+        if K == 1 or (vocab and b == len(sizes) - 1):
+            units[b] = [model.ranges[b]]
+            continue
+        r0, offs, off = model.ranges[b], [], 0
+        for (o, i) in bench.linears(h):
+            offs.append((off, o * i))
+            off += o * i
+        offs[-1] = (offs[-1][0], offs[-1][1] + (n - off))   # biases / LN with fc2
+        units[b] = [R.ratel_range(r0.param_bf16 + 2 * o, r0.grad_bf16 + 2 * o, 0, r0.master + 4 * o,
+                                  r0.exp_avg + 4 * o, r0.exp_avg_sq + 4 * o, ln, 1) for (o, ln) in offs]
+
+    def uid(b, j):
+        return b * K + j
+
+    def handoff_all(b, stream):
+        for j in range(len(units[b])):
+            R.ratel_offload_grad_chunk(uid(b, j), stream)
+
+    def wait_all(b, stream):
+        for j in range(len(units[b])):
+            R.ratel_block_wait(uid(b, j), stream)
     t_state = {"t": 1}
 
     def arm():
@@ -71,7 +99,7 @@ def run(args):
         with torch.cuda.stream(hi):
             if schedule == "opt":
                 for b in order:
-                    R.ratel_offload_grad_chunk(b, hi)
+                    handoff_all(b, hi)
                 arm()
             elif schedule == "bwd":
                 for b in order:
@@ -81,18 +109,21 @@ def run(args):
                     arm()
                 for j, b in enumerate(order):
                     if schedule != "deferred" and j >= args.ring:
-                        R.ratel_block_wait(b + args.ring, hi)   # ring slot free
-                    bw.block(b, b % args.ring)
-                    R.ratel_offload_grad_chunk(b, hi)
+                        wait_all(b + args.ring, hi)             # ring slot free
+                    if len(units[b]) > 1:                       # per-tensor hand-off
+                        bw.block(b, b % args.ring, on_linear=lambda k, b=b: R.ratel_offload_grad_chunk(uid(b, k), hi))
+                    else:
+                        bw.block(b, b % args.ring)
+                        R.ratel_offload_grad_chunk(uid(b, 0), hi)
                     if timeline:
                         tl["g"][b] = torch.cuda.Event(enable_timing=True)
                         tl["g"][b].record(hi)
                         if schedule != "deferred":
-                            R.ratel_block_wait(b, side)
+                            wait_all(b, side)
                             tl["d"][b] = torch.cuda.Event(enable_timing=True)
                             tl["d"][b].record(side)
                     if schedule == "naive" and args.residency == "device":
-                        R.ratel_block_wait(b, hi)               # handler not overlapped
+                        wait_all(b, hi)                         # handler not overlapped
                 if schedule == "deferred":
                     arm()
             if schedule != "bwd":
@@ -103,7 +134,8 @@ def run(args):
         cfg.staging = staging
         R.ratel_init(0, 0, 1, None, cfg)
         for b in range(len(sizes)):
-            R.ratel_register_block(b, [model.ranges[b]], res_code)
+            for j, r in enumerate(units[b]):
+                R.ratel_register_block(uid(b, j), [r], res_code)
         t_state["t"] = 1
 
     for tokens in args.tokens:
@@ -148,7 +180,8 @@ def run(args):
                               clk.get("power_w"))
                 R.ratel_finalize()
             tb = times["bwd"][0]
-            row = {"residency": args.residency, "tokens": tokens, "max_ctas": mc, "carveout": bool(args.carveout),
+            row = {"residency": args.residency, "granularity": args.granularity, "tokens": tokens, "max_ctas": mc,
+                   "carveout": bool(args.carveout),
                    "blocks": len(sizes),
                    "params": sum(sizes), "bwd_ms": tb, "bwd_tflops": 4 * sum(sizes) * tokens / (tb / 1e3) / 1e12}
             for sch, v in times.items():
@@ -180,4 +213,6 @@ if __name__ == "__main__":
     ap.add_argument("--warmup", type=int, default=1)
     ap.add_argument("--timeline", action="store_true", help="per-block grad-ready / update-done times")
     ap.add_argument("--carveout", action="store_true", help="cuBLAS SM carve-out = max_ctas for the backward")
+    ap.add_argument("--granularity", default="block", choices=["block", "tensor"],
+                    help="hand-off unit: a transformer block, or each of its four linears")
     run(ap.parse_args())
