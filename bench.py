@@ -214,7 +214,8 @@ def workload_config(args, world):
             "parallelism": (f"range-sharded x{world}" + (" (fused peer-store all-gather)" if args.fused_allgather else
                                                           " (NCCL all-gather)")) if world > 1 else "single GPU",
             "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
-            "max_grad_norm": args.clip, "update_streams": args.update_streams}
+            "max_grad_norm": args.clip, "update_streams": args.update_streams, "cta_tiles": args.cta_tiles,
+            "k1_kernel": ["tma", "ldg", "ldg_lite"][args.k1_kernel]}
 
 
 class PinnedArena:
@@ -664,6 +665,8 @@ def main():
     ap.add_argument("--overlap-tokens", type=int, default=8192, help="0 disables the AGO overlap probe")
     ap.add_argument("--arm", default="before", choices=["before", "after"],
                     help="arm before the hand-offs (AGO) or after the last one (deferred)")
+    ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
+    ap.add_argument("--k1-kernel", type=int, default=0, choices=[0, 1, 2], help="cfg.k1_kernel: 0 TMA, 1 LDG, 2 LDG_LITE")
     ap.add_argument("--tile-elems", type=int, default=0)
     ap.add_argument("--depth", type=int, default=0)
     ap.add_argument("--update-streams", type=int, default=2, choices=[1, 2],
@@ -717,6 +720,8 @@ def main():
         cfg.pipeline_depth = args.depth
     cfg.host_threads = args.host_threads
     cfg.update_streams = args.update_streams
+    cfg.cta_tiles = args.cta_tiles
+    cfg.k1_kernel = args.k1_kernel
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
     try:

@@ -114,6 +114,13 @@ typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1 } ratel
  * NCCL; clipping then uses the rank-local norm). */
 typedef enum { RATEL_COMM_AUTO = 0, RATEL_COMM_NONE = 1, RATEL_COMM_NCCL = 2 } ratel_comm;
 
+/* Update-kernel variants (same per-element arithmetic, bitwise-identical results):
+ * TMA      bulk-copy (TMA) shared-memory pipeline, one 224 KB CTA per SM, the fastest alone;
+ * LDG      register-staged 128/256-bit loads, 2 CTAs per SM, no shared memory;
+ * LDG_LITE register-staged, one octet in flight per thread, <= 64 registers, 4 CTAs per SM, no shared
+ *          memory: small enough to share an SM with a backward GEMM CTA while AGO overlaps them. */
+typedef enum { RATEL_UPDATE_TMA = 0, RATEL_UPDATE_LDG = 1, RATEL_UPDATE_LDG_LITE = 2 } ratel_k1_kernel;
+
 typedef struct {
   int mode;               /* ratel_mode; default RATEL_ADAMW */
   double max_grad_norm;   /* > 0 enables the global L2-norm clip (torch clip_grad_norm_); default 0 */
@@ -127,6 +134,14 @@ typedef struct {
   int update_streams;     /* device-residency updates alternate over this many low-priority streams,
                              1..2; default 2: block b+1's update starts on the SMs block b's tail
                              frees instead of after it (results are identical) */
+  int cta_tiles;          /* update-kernel tiles (4096 elements) per CTA.  0 (default): a persistent
+                             grid (one CTA per SM, max_ctas cap) taking tiles dynamically -- fastest
+                             alone.  > 0: a non-persistent grid of ceil(tiles / cta_tiles) CTAs, each
+                             retiring after its cta_tiles tiles, so kernels of higher-priority streams
+                             (the caller's backward) take SMs back within microseconds instead of
+                             waiting for a persistent CTA; max_ctas is ignored.  Results are identical. */
+  int k1_kernel;          /* ratel_k1_kernel: which update kernel (device-resident and tile updates);
+                             default RATEL_UPDATE_TMA.  Results are identical. */
 } ratel_config;
 
 /* One contiguous parameter range of a block (a flat tensor, or a block's

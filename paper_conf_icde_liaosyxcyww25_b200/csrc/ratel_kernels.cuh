@@ -76,6 +76,9 @@ struct UpdateParams {
   // counter only grows; one launch advances it by tiles + grid).
   unsigned long long* tile_ctr;
   unsigned long long tile_base;
+  // > 0: non-persistent grid, CTA b takes tiles [b*cta_tiles, (b+1)*cta_tiles)
+  // (tile_ctr is then NULL); 0: persistent grid.
+  uint32_t cta_tiles;
 };
 
 struct SumsqParams {
@@ -277,9 +280,12 @@ __device__ __forceinline__ double clip_coef_from(const double* sumsq, double max
 // K1.  Grid-stride over 8-element octets of each range, RATEL_K1_UNROLL
 // octets in flight per thread (all their loads issued before any math), then
 // the < 8-element scalar tail.
-template <int MODE, bool CLIP>
-__global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_kernel(const __grid_constant__ UpdateParams P) {
-  constexpr int U = RATEL_K1_UNROLL;
+// U / MINB: the default build (2 octets in flight, 2 CTAs/SM) or the "lite"
+// variant (cfg.k1_kernel = RATEL_UPDATE_LDG_LITE: 1 octet, 4 CTAs/SM, <= 64
+// registers, no shared memory) whose CTAs fit beside a backward GEMM CTA on
+// the same SM.
+template <int MODE, bool CLIP, int U = RATEL_K1_UNROLL, int MINB = RATEL_K1_MINB>
+__global__ void __launch_bounds__(kThreads, MINB) adam_update_kernel(const __grid_constant__ UpdateParams P) {
   const double coef_d = CLIP ? clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag) : 1.0;
   const float coef_f = static_cast<float>(coef_d);
   const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
@@ -439,14 +445,16 @@ __global__ void __launch_bounds__(kTmaThreads, RATEL_TMA_CTAS_PER_SM) adam_updat
       // measured in DESIGN.md §6).  The next grab is issued one tile early so
       // its latency overlaps the wait for a free stage.
       const bool dyn = P.tile_ctr != nullptr;
-      uint64_t k = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : blockIdx.x;
+      const uint64_t Y = P.cta_tiles;
+      uint64_t k = Y ? blockIdx.x * Y : dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : blockIdx.x;
+      const uint64_t lim = Y ? (k + Y < total ? k + Y : total) : total;
       int stage = 0;
       uint32_t phase = 0;
       for (;;) {
         uint64_t kn = k;
-        if (k < total) kn = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : k + gridDim.x;
+        if (k < lim) kn = Y ? k + 1 : dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : k + gridDim.x;
         mbar_wait(&empty[stage], phase ^ 1);
-        if (k >= total) {  // no more tiles: tell the consumers
+        if (k >= lim) {  // no more tiles: tell the consumers
           tile_id[stage] = ~0ull;
           mbar_arrive(&full[stage]);
           break;

@@ -150,7 +150,7 @@ struct Ctx {
   char sticky_msg[1024] = "";
   int device = 0, rank = 0, world = 1;
   ratel_config cfg{};
-  int sms = 0, k1_grid = 0, k2_grid = 0, rs_grid = 0;
+  int sms = 0, k1_grid = 0, k2_grid = 0, rs_grid = 0, lite_grid = 0;
   cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr, s_host = nullptr,
                s_tile = nullptr;
   // Device-residency update kernels alternate over s_k[0..update_streams-1];
@@ -273,19 +273,38 @@ int ctr_slot(cudaStream_t st) {
 
 template <int MODE, bool CLIP>
 void launch_k1(UpdateParams& P, unsigned grid, cudaStream_t st) {
+  if (G.cfg.k1_kernel == RATEL_UPDATE_LDG) {
+    adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(P);
+    return;
+  }
+  if (G.cfg.k1_kernel == RATEL_UPDATE_LDG_LITE) {
+    uint64_t max8 = 0;
+    for (int r = 0; r < P.nr; ++r) max8 = std::max<uint64_t>(max8, (P.r[r].n + 7) / 8);
+    const uint64_t want = std::max<uint64_t>(1, (max8 + kThreads - 1) / kThreads);
+    const unsigned g = static_cast<unsigned>(std::min<uint64_t>(want, static_cast<uint64_t>(G.lite_grid)));
+    adam_update_kernel<MODE, CLIP, 1, 4><<<g, kThreads, 0, st>>>(P);
+    return;
+  }
 #if RATEL_K1_TMA
   (void)grid;
   uint64_t tiles = 0;
   for (int r = 0; r < P.nr; ++r) tiles += ((P.r[r].n & ~7ull) + kTmaTile - 1) / kTmaTile;
   uint64_t cap = static_cast<uint64_t>(G.sms) * RATEL_TMA_CTAS_PER_SM;
   if (G.cfg.max_ctas > 0) cap = std::min<uint64_t>(cap, static_cast<uint64_t>(G.cfg.max_ctas));
-  const unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
+  unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
+  if (G.cfg.cta_tiles > 0) {  // non-persistent: CTA b takes tiles [b*Y, b*Y+Y), then retires
+    const uint64_t Y = static_cast<uint64_t>(G.cfg.cta_tiles);
+    P.cta_tiles = static_cast<uint32_t>(Y);
+    P.tile_ctr = nullptr;
+    g = static_cast<unsigned>(std::max<uint64_t>(1, (tiles + Y - 1) / Y));
+  } else {
 #if RATEL_TMA_DYNAMIC
-  const int slot = ctr_slot(st);
-  P.tile_ctr = G.d_ctr + slot;
-  P.tile_base = G.ctr_base[slot];
-  G.ctr_base[slot] += tiles + g;  // every tile taken once + one final grab per CTA
+    const int slot = ctr_slot(st);
+    P.tile_ctr = G.d_ctr + slot;
+    P.tile_base = G.ctr_base[slot];
+    G.ctr_base[slot] += tiles + g;  // every tile taken once + one final grab per CTA
 #endif
+  }
   adam_update_tma_kernel<MODE, CLIP><<<g, kTmaThreads, kTmaSmemBytes, st>>>(P);
 #else
   adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(P);
@@ -979,6 +998,9 @@ int validate_config(const ratel_config& c) {
     return set_error(RATEL_EINVAL, "cfg.comm");
   if (c.host_threads < 0) return set_error(RATEL_EINVAL, "cfg.host_threads must be >= 0");
   if (c.update_streams < 1 || c.update_streams > 2) return set_error(RATEL_EINVAL, "cfg.update_streams must be 1 or 2");
+  if (c.cta_tiles < 0) return set_error(RATEL_EINVAL, "cfg.cta_tiles must be >= 0");
+  if (c.k1_kernel != RATEL_UPDATE_TMA && c.k1_kernel != RATEL_UPDATE_LDG && c.k1_kernel != RATEL_UPDATE_LDG_LITE)
+    return set_error(RATEL_EINVAL, "cfg.k1_kernel");
   return RATEL_OK;
 }
 
@@ -1076,6 +1098,13 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK((prepare_k1<RATEL_ADAM_L2, false>()));
   CK((prepare_k1<RATEL_ADAM_L2, true>()));
   if (c.max_ctas > 0) G.k1_grid = std::min(G.k1_grid, c.max_ctas);
+  int occ_lite = 0;
+  if (c.mode == RATEL_ADAMW)
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_lite, adam_update_kernel<RATEL_ADAMW, false, 1, 4>, kThreads, 0));
+  else
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ_lite, adam_update_kernel<RATEL_ADAM_L2, false, 1, 4>, kThreads, 0));
+  G.lite_grid = G.sms * std::max(occ_lite, 1);
+  if (c.max_ctas > 0) G.lite_grid = std::min(G.lite_grid, c.max_ctas);
   G.k2_grid = G.sms * 4;
   CK(cudaMalloc(&G.d_ctr, 5 * sizeof(unsigned long long)));
   CK(cudaMemset(G.d_ctr, 0, 5 * sizeof(unsigned long long)));
@@ -1122,6 +1151,8 @@ void ratel_default_config(ratel_config* cfg) {
   cfg->comm = RATEL_COMM_AUTO;
   cfg->host_threads = 0;
   cfg->update_streams = 2;
+  cfg->cta_tiles = 0;
+  cfg->k1_kernel = RATEL_UPDATE_TMA;
 }
 
 uint64_t ratel_padded_numel(uint64_t numel, int world_size) {

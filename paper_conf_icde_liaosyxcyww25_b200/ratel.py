@@ -36,6 +36,9 @@ RATEL_STAGING_SERIALIZED = 1
 RATEL_COMM_AUTO = 0
 RATEL_COMM_NONE = 1
 RATEL_COMM_NCCL = 2
+RATEL_UPDATE_TMA = 0
+RATEL_UPDATE_LDG = 1
+RATEL_UPDATE_LDG_LITE = 2
 RATEL_MAX_BLOCKS = 4096
 RATEL_MAX_RANGES_PER_BLOCK = 32
 
@@ -62,6 +65,8 @@ class ratel_config(ctypes.Structure):
         ("comm", ctypes.c_int),
         ("host_threads", ctypes.c_int),
         ("update_streams", ctypes.c_int),
+        ("cta_tiles", ctypes.c_int),
+        ("k1_kernel", ctypes.c_int),
     ]
 
 

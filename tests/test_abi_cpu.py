@@ -77,8 +77,8 @@ def test_init_without_gpu_fails_cleanly():
 def test_default_config():
     c = R.ratel_default_config()
     assert (c.mode, c.max_grad_norm, c.pipeline_depth, c.staging, c.tile_elems, c.max_ctas, c.timing, c.comm,
-            c.host_threads, c.update_streams) == \
-        (R.RATEL_ADAMW, 0.0, 4, R.RATEL_STAGING_PIPELINED, 1 << 24, 0, 0, R.RATEL_COMM_AUTO, 0, 2)
+            c.host_threads, c.update_streams, c.cta_tiles, c.k1_kernel) == \
+        (R.RATEL_ADAMW, 0.0, 4, R.RATEL_STAGING_PIPELINED, 1 << 24, 0, 0, R.RATEL_COMM_AUTO, 0, 2, 0, R.RATEL_UPDATE_TMA)
 
 
 @pytest.mark.parametrize("world", [1, 2, 3, 4, 8])
@@ -117,8 +117,9 @@ def test_generator_keys_match_synth():
 
 
 def test_struct_layouts_match_header():
-    # ratel_config: int, double, int, int, uint64, int, int, int, int, int -> 56 bytes
-    assert ctypes.sizeof(R.ratel_config) == 56
+    # ratel_config: int, double, int, int, uint64, int x 7 -> 64 bytes
+    assert ctypes.sizeof(R.ratel_config) == 64
+    assert R.ratel_config.k1_kernel.offset == 56
     assert R.ratel_config.update_streams.offset == 48
     assert R.ratel_config.tile_elems.offset == 24
     # ratel_range: 2 ptrs, int, 3 ptrs, uint64, int -> 64 bytes

@@ -182,6 +182,38 @@ def test_max_ctas_cap_bitwise(cuda_dev, max_ctas):
     assert_bitwise(snapshot(a), snapshot(b))
 
 
+@pytest.mark.parametrize("cta_tiles,clip", [(1, 0.0), (3, 0.0), (8, 0.05), (1000, 0.0)])
+def test_cta_tiles_nonpersistent_grid_bitwise(cuda_dev, cta_tiles, clip):
+    """cfg.cta_tiles > 0: a non-persistent grid whose CTAs retire after
+    cta_tiles tiles (ragged last CTA, tiles crossing range boundaries, one CTA
+    covering everything at 1000) must update every element exactly as the
+    persistent grid does, also in clip mode, and match the oracle."""
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 2, check_every=False, max_norm=clip)
+    b = _fresh(SIZES, cuda_dev)
+    run(b, 2, max_norm=clip, cta_tiles=cta_tiles)
+    assert_bitwise(snapshot(a), snapshot(b))
+
+
+@pytest.mark.parametrize("kernel,max_ctas", [(1, 0), (2, 0), (2, 5)])
+def test_k1_kernel_variants_bitwise(cuda_dev, kernel, max_ctas):
+    """cfg.k1_kernel = LDG / LDG_LITE (register-staged, no shared memory)
+    gives the TMA kernel's bits and matches the oracle (also capped)."""
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 2, check_every=False)
+    b = _fresh(SIZES, cuda_dev)
+    run(b, 2, k1_kernel=kernel, max_ctas=max_ctas)
+    assert_bitwise(snapshot(a), snapshot(b))
+
+
+def test_cta_tiles_pinned_host_bitwise(cuda_dev):
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 2, check_every=False)
+    b = _fresh(SIZES, cuda_dev, pinned=True)
+    run(b, 2, check_every=False, tile_elems=65_536, cta_tiles=2)
+    assert_bitwise(snapshot(a), snapshot(b))
+
+
 def test_large_block_ring_wraps_vs_oracle(cuda_dev):
     """20M + 5 elements, two ranges: ~33 tiles per CTA at the full grid."""
     b = GpuBlock(0, [20_000_005, 4_096 * 7 + 3], cuda_dev)

@@ -52,7 +52,7 @@ def run(args):
     ring = model.grad_ring
     res_code = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
     vocab = bench.VOCAB if len(sizes) == L + 1 else 0
-    hi = torch.cuda.Stream(priority=-2)
+    hi = torch.cuda.Stream(priority=args.bwd_priority)
     order = list(reversed(range(len(sizes))))
     # --granularity tensor: every linear of a block (its weights; the last one
     # also carries the block's 13h biases/LN) is its own registered unit,
@@ -131,6 +131,8 @@ def run(args):
 
     def init(mc, staging):
         cfg.max_ctas = mc
+        cfg.cta_tiles = args.cta_tiles
+        cfg.k1_kernel = args.k1_kernel
         cfg.staging = staging
         R.ratel_init(0, 0, 1, None, cfg)
         for b in range(len(sizes)):
@@ -180,7 +182,9 @@ def run(args):
                               clk.get("power_w"))
                 R.ratel_finalize()
             tb = times["bwd"][0]
-            row = {"residency": args.residency, "granularity": args.granularity, "tokens": tokens, "max_ctas": mc,
+            row = {"residency": args.residency, "granularity": args.granularity, "cta_tiles": args.cta_tiles,
+                   "k1_kernel": args.k1_kernel, "bwd_priority": args.bwd_priority, "ring": args.ring,
+                   "tokens": tokens, "max_ctas": mc,
                    "carveout": bool(args.carveout),
                    "blocks": len(sizes),
                    "params": sum(sizes), "bwd_ms": tb, "bwd_tflops": 4 * sum(sizes) * tokens / (tb / 1e3) / 1e12}
@@ -213,6 +217,10 @@ if __name__ == "__main__":
     ap.add_argument("--warmup", type=int, default=1)
     ap.add_argument("--timeline", action="store_true", help="per-block grad-ready / update-done times")
     ap.add_argument("--carveout", action="store_true", help="cuBLAS SM carve-out = max_ctas for the backward")
+    ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
+    ap.add_argument("--k1-kernel", type=int, default=0, help="cfg.k1_kernel: 0 TMA, 1 LDG, 2 LDG_LITE")
+    ap.add_argument("--bwd-priority", type=int, default=-2,
+                    help="torch stream priority of the synthetic backward (0 = default streams = the optimizer's)")
     ap.add_argument("--granularity", default="block", choices=["block", "tensor"],
                     help="hand-off unit: a transformer block, or each of its four linears")
     run(ap.parse_args())
