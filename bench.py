@@ -435,6 +435,87 @@ def overlap_probe(args, R, torch, dev, model, sizes, order, t0):
 HOST_ENQUEUE_MS = []   # host time to issue one step (arm + hand-offs + stream sync)
 
 
+def overlap_host_probe(args, R, torch, dev, dev_index):
+    """The north star's host-resident overlap target (Fig. 7 analog): pinned-host
+    states of `--overlap-host-blocks` 13B blocks, each of a block's four linears
+    registered as its own unit and handed off right after its dW GEMM (the
+    paper's per-tensor hand-off), with a synthetic backward of
+    `--overlap-host-tokens` tokens.  Exposed = AGO step - backward alone."""
+    L, h = SHAPES[args.shape]
+    sizes = model_blocks(args.shape, with_embedding=False)[:args.overlap_host_blocks]
+    cfg = R.ratel_default_config()
+    R.ratel_init(dev_index, 0, 1, None, cfg)
+    model = Model(R, torch, dev, sizes, 1, 0, "host", grad_ring=3)
+    R.ratel_finalize()
+    units = []
+    for b, n in enumerate(sizes):
+        r0, offs, off = model.ranges[b], [], 0
+        for (o, i) in linears(h):
+            offs.append([off, o * i])
+            off += o * i
+        offs[-1][1] += n - off            # biases / LN ride with fc2
+        units.append([R.ratel_range(r0.param_bf16 + 2 * o, r0.grad_bf16 + 2 * o, 0, r0.master + 4 * o,
+                                    r0.exp_avg + 4 * o, r0.exp_avg_sq + 4 * o, ln, 1) for o, ln in offs])
+    K = 4
+    R.ratel_init(dev_index, 0, 1, None, cfg)
+    try:
+        for b in range(len(sizes)):
+            for j, r in enumerate(units[b]):
+                R.ratel_register_block(b * K + j, [r], R.RATEL_PINNED_HOST)
+        bw = SynthBackward(dev, h, args.overlap_host_tokens, model.p16, model.grad_ring, 0)
+        s = torch.cuda.Stream(device=dev, priority=-2)
+        order = list(reversed(range(len(sizes))))
+        t = [1]
+
+        def bwd():
+            with torch.cuda.stream(s):
+                for b in order:
+                    bw.block(b, b % 3)
+
+        def opt():
+            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+            t[0] += 1
+            for b in order:
+                for j in range(K):
+                    R.ratel_offload_grad_chunk(b * K + j, s)
+            R.ratel_sync(s)
+
+        def ago():
+            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+            t[0] += 1
+            with torch.cuda.stream(s):
+                for jb, b in enumerate(order):
+                    if jb >= 3:
+                        for j in range(K):
+                            R.ratel_block_wait((b + 3) * K + j, s)   # ring slot consumed
+                    bw.block(b, b % 3, on_linear=lambda j, b=b: R.ratel_offload_grad_chunk(b * K + j, s))
+            R.ratel_sync(s)
+
+        res = {}
+        for name, fn in (("bwd", bwd), ("opt", opt), ("ago", ago)):
+            fn()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            for _ in range(2):
+                fn()
+            e1.record(s)
+            e1.synchronize()
+            res[name] = e0.elapsed_time(e1) / 2
+        P = sum(sizes)
+        return {"tokens": args.overlap_host_tokens, "blocks": len(sizes), "params": P,
+                "residency": "pinned-host", "handoff": "per tensor (4 linears per block)",
+                "backward_ms": res["bwd"], "optimizer_alone_ms": res["opt"], "ago_step_ms": res["ago"],
+                "exposed_optimizer_ms": res["ago"] - res["bwd"],
+                "hidden_fraction": 1.0 - (res["ago"] - res["bwd"]) / res["opt"],
+                "host_link_gbs_optimizer_alone": 24 * P / (res["opt"] / 1e3) / 1e9,
+                "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)"}
+    finally:
+        R.ratel_finalize()
+        del model
+        torch.cuda.empty_cache()
+
+
 def timed_steps(R, torch, order, stream, t0, K, pre_step=None, post_step=None):
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ev0.record(stream)
@@ -663,6 +744,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--oracle-sample", type=int, default=1 << 25)
     ap.add_argument("--overlap-tokens", type=int, default=8192, help="0 disables the AGO overlap probe")
+    ap.add_argument("--overlap-host-tokens", type=int, default=131072,
+                    help="pinned-host per-tensor AGO overlap probe (0 disables)")
+    ap.add_argument("--overlap-host-blocks", type=int, default=8)
     ap.add_argument("--arm", default="before", choices=["before", "after"],
                     help="arm before the hand-offs (AGO) or after the last one (deferred)")
     ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
@@ -822,6 +906,14 @@ def main():
         if e2e is None:
             e2e = e2e_host
 
+        overlap_host = None
+        if args.overlap_host_tokens > 0 and world == 1 and args.residency == "device":
+            try:
+                overlap_host = overlap_host_probe(args, R, torch, dev, local)
+            except Exception as ex:  # report, do not hide
+                overlap_host = {"error": repr(ex)[:300]}
+            torch.cuda.empty_cache()
+
         cpu = None
         if rank == 0 and world == 1 and not args.no_cpu_baseline:
             n = args.oracle_sample
@@ -841,7 +933,7 @@ def main():
                     # first timed step: issued into a drained launch queue, so this is the
                     # host cost of a step (later ones wait on queue back-pressure)
                     "host_enqueue_ms_first_step": HOST_ENQUEUE_MS[0] if HOST_ENQUEUE_MS else None,
-                    "overlap": overlap,
+                    "overlap": overlap, "overlap_host": overlap_host,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
             print(json.dumps(line), flush=True)
     finally:

@@ -91,8 +91,8 @@ class Ratel_Optimizer:
     own unit (and the block's no-decay parameters as one more), each handed
     off as soon as its own gradient is complete -- the paper's per-tensor
     handler.  Finer units shorten the update tail after the
-    last gradient (pinned-host 13B blocks at 98K tokens: 38 ms exposed vs 98 ms,
-    profiles/r01_overlap_granularity.jsonl); the result is bitwise the same.
+    last gradient (a block's update done 12-13 ms after its last gradient instead
+    of ~70 ms, profiles/r01_overlap_granularity.jsonl); the result is bitwise the same.
     `blocks`/`block_ids`/`state(i)` then index units."""
 
     def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,

@@ -133,6 +133,8 @@ def run(args):
         cfg.max_ctas = mc
         cfg.cta_tiles = args.cta_tiles
         cfg.k1_kernel = args.k1_kernel
+        if args.tile_elems:
+            cfg.tile_elems = args.tile_elems
         cfg.staging = staging
         R.ratel_init(0, 0, 1, None, cfg)
         for b in range(len(sizes)):
@@ -184,6 +186,7 @@ def run(args):
             tb = times["bwd"][0]
             row = {"residency": args.residency, "granularity": args.granularity, "cta_tiles": args.cta_tiles,
                    "k1_kernel": args.k1_kernel, "bwd_priority": args.bwd_priority, "ring": args.ring,
+                   "tile_elems": args.tile_elems,
                    "tokens": tokens, "max_ctas": mc,
                    "carveout": bool(args.carveout),
                    "blocks": len(sizes),
@@ -219,6 +222,7 @@ if __name__ == "__main__":
     ap.add_argument("--carveout", action="store_true", help="cuBLAS SM carve-out = max_ctas for the backward")
     ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
     ap.add_argument("--k1-kernel", type=int, default=0, help="cfg.k1_kernel: 0 TMA, 1 LDG, 2 LDG_LITE")
+    ap.add_argument("--tile-elems", type=int, default=0, help="cfg.tile_elems (pinned-host tile ring)")
     ap.add_argument("--bwd-priority", type=int, default=-2,
                     help="torch stream priority of the synthetic backward (0 = default streams = the optimizer's)")
     ap.add_argument("--granularity", default="block", choices=["block", "tensor"],
