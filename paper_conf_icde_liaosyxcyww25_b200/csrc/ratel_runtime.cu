@@ -80,8 +80,9 @@ struct Block {
   std::vector<ratel_range> ranges;
   std::vector<Slice> slices;
   cudaEvent_t ev_grad = nullptr;  // "gradient arrived" -- recorded on the caller's stream
-  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt (s_host for HOST_COMPUTE)
+  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt (s_h2d for HOST_COMPUTE)
   cudaEvent_t ev_gh = nullptr;    // HOST_COMPUTE: G16 slices landed in host staging
+  cudaEvent_t ev_hc = nullptr;    // HOST_COMPUTE: the CPU update of this block finished (on s_host)
   std::vector<uint16_t*> h_g, h_p;  // HOST_COMPUTE: pinned G16 / P16 staging per range (rank slice)
   std::vector<std::vector<uint16_t*>> peers;  // per range: every rank's P16 base as mapped here (fused all-gather)
   // Fused data-parallel gradient reduction (R17): per range, every rank's
@@ -588,14 +589,18 @@ int enqueue_host_compute(Block& B) {
     delete task;
     return sticky_fail(RATEL_ECUDA, "host handler enqueue failed: %s", cudaGetErrorString(e));
   }
+  // P16 host->device on the H2D stream, so the host stream goes straight on to
+  // the next block's CPU update while this block's P16 crosses the link.
+  CK(cudaEventRecord(B.ev_hc, G.s_host));
+  CK(cudaStreamWaitEvent(G.s_h2d, B.ev_hc, 0));
   for (size_t i = 0; i < B.ranges.size(); ++i) {
     const Slice& s = B.slices[i];
     const uint64_t n = s.end - s.begin;
     if (n == 0) continue;
     CK(cudaMemcpyAsync(static_cast<uint16_t*>(B.ranges[i].param_bf16) + s.begin, B.h_p[i], n * 2,
-                       cudaMemcpyHostToDevice, G.s_host));
+                       cudaMemcpyHostToDevice, G.s_h2d));
   }
-  CK(cudaEventRecord(B.ev_done, G.s_host));
+  CK(cudaEventRecord(B.ev_done, G.s_h2d));
   return RATEL_OK;
 }
 
@@ -1021,6 +1026,7 @@ void destroy_all() {
     if (B.ev_grad) cudaEventDestroy(B.ev_grad);
     if (B.ev_done) cudaEventDestroy(B.ev_done);
     if (B.ev_gh) cudaEventDestroy(B.ev_gh);
+    if (B.ev_hc) cudaEventDestroy(B.ev_hc);
     if (B.ev_ready) cudaEventDestroy(B.ev_ready);
     if (B.ev_rel) cudaEventDestroy(B.ev_rel);
     for (uint16_t* p : B.h_g) cudaFreeHost(p);
@@ -1284,6 +1290,7 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
       CK(cudaHostAlloc(&B.h_p[i], n * 2, cudaHostAllocDefault));
     }
     CK(cudaEventCreateWithFlags(&B.ev_gh, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&B.ev_hc, cudaEventDisableTiming));
   }
   if (residency == RATEL_SSD) {
     if (G.ssd == nullptr) RK(ssd_create());
