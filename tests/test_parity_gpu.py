@@ -457,6 +457,40 @@ def test_fullsize_13b_blocks_sampled_vs_oracle(cuda_dev):
             assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
 
 
+def test_range_beyond_2pow32_elements_sampled_vs_oracle(cuda_dev):
+    """Maximum sizes: one range of 2^32 + 4099 elements (69 GB of states and
+    grads in HBM), so tile indices, element offsets and the generator's
+    counters cross 2^31 and 2^32 (64-bit indexing everywhere) and the range
+    ends in a ragged scalar tail.  Two steps; sampled elements around both
+    boundaries and the tail vs the oracle; P16 == bf16(P32) on the samples."""
+    n = (1 << 32) + 4099
+    picks = [np.arange(0, 32), np.arange((1 << 31) - 40, (1 << 31) + 40), np.arange((1 << 32) - 40, (1 << 32) + 40),
+             np.arange(n - 40, n), np.random.default_rng(5).integers(0, n, 50_000)]
+    idx = np.unique(np.concatenate(picks)).astype(np.uint64)
+    with ratel_lib():
+        th = torch.empty(n, dtype=torch.float32, device=cuda_dev)
+        R.ratel_gen_theta0(th.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, 0))
+        m = torch.zeros(n, device=cuda_dev)
+        v = torch.zeros(n, device=cuda_dev)
+        p = torch.zeros(R.ratel_padded_numel(n, 1), dtype=torch.bfloat16, device=cuda_dev)
+        g = torch.empty(R.ratel_padded_numel(n, 1), dtype=torch.bfloat16, device=cuda_dev)
+        R.ratel_register_block(0, [R.make_range(p, g, th, m, v, n)], R.RATEL_DEVICE)
+        ref = oracle.Range.fresh(synth.theta0_at(idx, block=0))
+        for t in (1, 2):
+            R.ratel_gen_grad16(g.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, 0))
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            R.ratel_offload_grad_chunk(0, None)
+            R.ratel_sync(None)
+            oracle.adam_range(ref, synth.grad16_at(idx, step=t, block=0), oracle.hparams(step=t))
+        ii = torch.from_numpy(idx.astype(np.int64)).to(cuda_dev)
+        got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
+                   p16=torch_to_u16(p[ii]))
+        check_range(got, ref, own_rne=oracle.bf16_rne, what="2^32+ range")
+        assert np.array_equal(got["p16"], oracle.bf16_rne(got["p32"]))
+    del th, m, v, p, g
+    torch.cuda.empty_cache()
+
+
 def test_max_ranges_and_block_ids(cuda_dev):
     """A block with RATEL_MAX_RANGES_PER_BLOCK ranges (sizes 1..., mixed wd
     flags) under the largest block id, next to a one-range block; and the
