@@ -215,7 +215,7 @@ def workload_config(args, world):
                                                           " (NCCL all-gather)")) if world > 1 else "single GPU",
             "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
             "max_grad_norm": args.clip, "update_streams": args.update_streams, "cta_tiles": args.cta_tiles,
-            "k1_kernel": ["tma", "ldg", "ldg_lite"][args.k1_kernel]}
+            "k1_kernel": ["tma", "ldg", "ldg_lite"][args.k1_kernel], "staging": args.staging}
 
 
 class PinnedArena:
@@ -750,6 +750,8 @@ def main():
     ap.add_argument("--arm", default="before", choices=["before", "after"],
                     help="arm before the hand-offs (AGO) or after the last one (deferred)")
     ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
+    ap.add_argument("--staging", default="pipelined", choices=["pipelined", "serialized", "zero_copy"],
+                    help="pinned-host residency: tile ring (Fig. 3b / 3a) or in-place over the link")
     ap.add_argument("--k1-kernel", type=int, default=0, choices=[0, 1, 2], help="cfg.k1_kernel: 0 TMA, 1 LDG, 2 LDG_LITE")
     ap.add_argument("--tile-elems", type=int, default=0)
     ap.add_argument("--depth", type=int, default=0)
@@ -805,6 +807,8 @@ def main():
     cfg.host_threads = args.host_threads
     cfg.update_streams = args.update_streams
     cfg.cta_tiles = args.cta_tiles
+    cfg.staging = {"pipelined": R.RATEL_STAGING_PIPELINED, "serialized": R.RATEL_STAGING_SERIALIZED,
+                   "zero_copy": R.RATEL_STAGING_ZERO_COPY}[args.staging]
     cfg.k1_kernel = args.k1_kernel
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None

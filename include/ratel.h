@@ -104,8 +104,12 @@ typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
  * update of tile k and write-back of tile k-1 overlap on three streams; the
  * tile updates run on a high-priority stream so they slot in between
  * backward kernels);
- * SERIALIZED = Fig. 3a (naive AGO: stage-in, update, write-back in series). */
-typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1 } ratel_staging;
+ * SERIALIZED = Fig. 3a (naive AGO: stage-in, update, write-back in series);
+ * ZERO_COPY = no tiles: the register-staged update kernel (RATEL_UPDATE_LDG_LITE)
+ * reads and writes the page-locked states in place over the host link
+ * (unified addressing), one kernel per range; grid = cfg.max_ctas if set.
+ * Results are identical in all three. */
+typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1, RATEL_STAGING_ZERO_COPY = 2 } ratel_staging;
 
 /* Collectives: AUTO = NCCL when world_size > 1; NCCL = also for world_size 1
  * (a one-rank communicator: exercises the NCCL calls on one GPU); NONE = no

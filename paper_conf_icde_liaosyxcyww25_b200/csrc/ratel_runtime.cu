@@ -273,12 +273,12 @@ int ctr_slot(cudaStream_t st) {
 }
 
 template <int MODE, bool CLIP>
-void launch_k1(UpdateParams& P, unsigned grid, cudaStream_t st) {
-  if (G.cfg.k1_kernel == RATEL_UPDATE_LDG) {
+void launch_k1(UpdateParams& P, unsigned grid, cudaStream_t st, int kernel) {
+  if (kernel == RATEL_UPDATE_LDG) {
     adam_update_kernel<MODE, CLIP><<<grid, kThreads, 0, st>>>(P);
     return;
   }
-  if (G.cfg.k1_kernel == RATEL_UPDATE_LDG_LITE) {
+  if (kernel == RATEL_UPDATE_LDG_LITE) {
     uint64_t max8 = 0;
     for (int r = 0; r < P.nr; ++r) max8 = std::max<uint64_t>(max8, (P.r[r].n + 7) / 8);
     const uint64_t want = std::max<uint64_t>(1, (max8 + kThreads - 1) / kThreads);
@@ -339,8 +339,10 @@ void launch_k1_rs(RsUpdateParams& Q, unsigned grid, cudaStream_t st) {
 }
 
 // gp != nullptr: the fused-reduction kernel (gp[i] = the rank grads of rd[i]).
+// kernel: ratel_k1_kernel to use, -1 = cfg.k1_kernel.
 int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* pd = nullptr,
-                  const GradPeers* gp = nullptr) {
+                  const GradPeers* gp = nullptr, int kernel = -1) {
+  if (kernel < 0) kernel = G.cfg.k1_kernel;
   if (nr == 0) return RATEL_OK;
   std::lock_guard<std::mutex> lk(g_launch_mu);
   UpdateParams P{};
@@ -383,9 +385,9 @@ int launch_update(const RangeDesc* rd, int nr, cudaStream_t st, const PeerDesc* 
     else
       clip ? launch_k1_rs<RATEL_ADAM_L2, true>(Q, grid, st) : launch_k1_rs<RATEL_ADAM_L2, false>(Q, grid, st);
   } else if (G.cfg.mode == RATEL_ADAMW) {
-    clip ? launch_k1<RATEL_ADAMW, true>(P, grid, st) : launch_k1<RATEL_ADAMW, false>(P, grid, st);
+    clip ? launch_k1<RATEL_ADAMW, true>(P, grid, st, kernel) : launch_k1<RATEL_ADAMW, false>(P, grid, st, kernel);
   } else {
-    clip ? launch_k1<RATEL_ADAM_L2, true>(P, grid, st) : launch_k1<RATEL_ADAM_L2, false>(P, grid, st);
+    clip ? launch_k1<RATEL_ADAM_L2, true>(P, grid, st, kernel) : launch_k1<RATEL_ADAM_L2, false>(P, grid, st, kernel);
   }
   CK(cudaGetLastError());
   ++G.launches;
@@ -466,6 +468,31 @@ PeerDesc peer_desc(const Block& B, size_t i, uint64_t off) {
 bool has_peers(const Block& B, size_t i) { return i < B.peers.size() && !B.peers[i].empty(); }
 
 // One staged tile of a pinned-host range: H2D(theta, m, v) -> K1 -> D2H.
+// RATEL_STAGING_ZERO_COPY: the register-staged update kernel reads and
+// writes the range's page-locked host states in place (unified addressing:
+// the host pointer is a valid device address), so theta/m/v cross the host
+// link exactly once each way with no device tiles, copy engines or extra HBM
+// traffic; the grid is cfg.max_ctas (default all SMs x the lite kernel's
+// occupancy) of no-shared-memory CTAs.
+int update_in_place_over_link(const Block& B, size_t ri) {
+  const ratel_range& r = B.ranges[ri];
+  const Slice& s = B.slices[ri];
+  const uint64_t n = s.end - s.begin;
+  if (n == 0) return RATEL_OK;
+  RangeDesc rd{};
+  rd.g = grad_ptr(r, s);
+  rd.th = r.master;
+  rd.m = r.exp_avg;
+  rd.v = r.exp_avg_sq;
+  rd.p = static_cast<uint16_t*>(r.param_bf16) + s.begin;
+  rd.n = n;
+  rd.wd_on = r.apply_weight_decay != 0;
+  GradPeers gp{};
+  if (B.rs) gp = grad_peers(B, ri, 0);
+  const PeerDesc pd = peer_desc(B, ri, 0);
+  return launch_update(&rd, 1, G.s_tile, &pd, B.rs ? &gp : nullptr, RATEL_UPDATE_LDG_LITE);
+}
+
 int stage_tile(const Block& B, size_t ri, uint64_t off, uint64_t len) {
   Nvtx nv("ratel tile %llu", static_cast<unsigned long long>(G.ring_k));
   const ratel_range& r = B.ranges[ri];
@@ -931,6 +958,10 @@ int enqueue_block(Block& B, const std::vector<cudaEvent_t>* ssd_wait = nullptr) 
     for (size_t i = 0; i < B.ranges.size(); ++i) {
       const Slice& s = B.slices[i];
       const uint64_t n = s.end - s.begin;
+      if (G.cfg.staging == RATEL_STAGING_ZERO_COPY) {
+        RK(update_in_place_over_link(B, i));
+        continue;
+      }
       for (uint64_t off = 0; off < n; off += G.cfg.tile_elems)
         RK(stage_tile(B, i, off, std::min<uint64_t>(G.cfg.tile_elems, n - off)));
     }
@@ -995,7 +1026,8 @@ int validate_config(const ratel_config& c) {
     return set_error(RATEL_EINVAL, "cfg.max_grad_norm must be finite and >= 0");
   if (c.pipeline_depth < 2 || c.pipeline_depth > kMaxDepth)
     return set_error(RATEL_EINVAL, "cfg.pipeline_depth must be in [2, %d]", kMaxDepth);
-  if (c.staging != RATEL_STAGING_PIPELINED && c.staging != RATEL_STAGING_SERIALIZED)
+  if (c.staging != RATEL_STAGING_PIPELINED && c.staging != RATEL_STAGING_SERIALIZED &&
+      c.staging != RATEL_STAGING_ZERO_COPY)
     return set_error(RATEL_EINVAL, "cfg.staging");
   if (c.tile_elems == 0 || (c.tile_elems & 7u)) return set_error(RATEL_EINVAL, "cfg.tile_elems must be a positive multiple of 8");
   if (c.max_ctas < 0) return set_error(RATEL_EINVAL, "cfg.max_ctas must be >= 0");

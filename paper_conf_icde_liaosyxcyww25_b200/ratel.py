@@ -33,6 +33,7 @@ RATEL_ADAMW = 0
 RATEL_ADAM_L2 = 1
 RATEL_STAGING_PIPELINED = 0
 RATEL_STAGING_SERIALIZED = 1
+RATEL_STAGING_ZERO_COPY = 2
 RATEL_COMM_AUTO = 0
 RATEL_COMM_NONE = 1
 RATEL_COMM_NCCL = 2

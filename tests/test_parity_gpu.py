@@ -162,7 +162,8 @@ def test_bitwise_handoff_order_and_deferred(cuda_dev):
     assert_bitwise(sa, snapshot(c))
 
 
-@pytest.mark.parametrize("depth,staging,tile", [(2, 0, 4096), (3, 0, 65_536), (3, 1, 8192), (2, 0, 1 << 24)])
+@pytest.mark.parametrize("depth,staging,tile", [(2, 0, 4096), (3, 0, 65_536), (3, 1, 8192), (2, 0, 1 << 24),
+                                                (2, 2, 4096)])
 def test_pinned_host_bitwise_equals_device(cuda_dev, depth, staging, tile):
     a = _fresh(SIZES, cuda_dev)
     run(a, 3, check_every=False)
@@ -203,6 +204,19 @@ def test_k1_kernel_variants_bitwise(cuda_dev, kernel, max_ctas):
     run(a, 2, check_every=False)
     b = _fresh(SIZES, cuda_dev)
     run(b, 2, k1_kernel=kernel, max_ctas=max_ctas)
+    assert_bitwise(snapshot(a), snapshot(b))
+
+
+@pytest.mark.parametrize("mode,max_norm,max_ctas", [(oracle.ADAMW, 0.0, 0), (oracle.ADAM_L2, 0.05, 0),
+                                                     (oracle.ADAMW, 0.05, 3)])
+def test_zero_copy_staging_vs_oracle(cuda_dev, mode, max_norm, max_ctas):
+    """RATEL_STAGING_ZERO_COPY: the update kernel reads/writes the pinned
+    host states in place over the link; oracle parity (clip, Adam-L2, a
+    3-CTA grid cycling many times) and bitwise = device residency."""
+    a = _fresh(SIZES, cuda_dev)
+    run(a, 3, mode=mode, max_norm=max_norm, check_every=False)
+    b = _fresh(SIZES, cuda_dev, pinned=True)
+    run(b, 3, mode=mode, max_norm=max_norm, staging=2, max_ctas=max_ctas)
     assert_bitwise(snapshot(a), snapshot(b))
 
 

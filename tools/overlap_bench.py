@@ -154,7 +154,7 @@ def run(args):
                 if sch == "deferred" and args.ring < len(sizes):
                     continue
                 staging = R.RATEL_STAGING_SERIALIZED if (sch == "naive" and args.residency == "host") \
-                    else R.RATEL_STAGING_PIPELINED
+                    else (R.RATEL_STAGING_ZERO_COPY if args.zero_copy else R.RATEL_STAGING_PIPELINED)
                 init(mc, staging)
                 for _ in range(args.warmup):
                     one(sch, bw)
@@ -186,7 +186,7 @@ def run(args):
             tb = times["bwd"][0]
             row = {"residency": args.residency, "granularity": args.granularity, "cta_tiles": args.cta_tiles,
                    "k1_kernel": args.k1_kernel, "bwd_priority": args.bwd_priority, "ring": args.ring,
-                   "tile_elems": args.tile_elems,
+                   "tile_elems": args.tile_elems, "zero_copy": bool(args.zero_copy),
                    "tokens": tokens, "max_ctas": mc,
                    "carveout": bool(args.carveout),
                    "blocks": len(sizes),
@@ -223,6 +223,7 @@ if __name__ == "__main__":
     ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
     ap.add_argument("--k1-kernel", type=int, default=0, help="cfg.k1_kernel: 0 TMA, 1 LDG, 2 LDG_LITE")
     ap.add_argument("--tile-elems", type=int, default=0, help="cfg.tile_elems (pinned-host tile ring)")
+    ap.add_argument("--zero-copy", action="store_true", help="pinned-host: RATEL_STAGING_ZERO_COPY")
     ap.add_argument("--bwd-priority", type=int, default=-2,
                     help="torch stream priority of the synthetic backward (0 = default streams = the optimizer's)")
     ap.add_argument("--granularity", default="block", choices=["block", "tensor"],
