@@ -49,8 +49,40 @@ def Ratel_init(device: int | None = None, **cfg_kw):
         R.ratel_finalize()
 
 
+class _SsdFile:
+    """One state file for every SSD range of an optimizer: ranges are laid out
+    back to back (ratel_ssd_range_bytes each).  Written through a buffered fd
+    (theta0, zeros), handed to the library as an O_DIRECT fd."""
+
+    def __init__(self, path):
+        import os
+        self.path = path
+        self.size = 0
+        self.fd_buf = os.open(path, os.O_RDWR | os.O_CREAT | os.O_TRUNC, 0o600)
+        self.fd = None
+
+    def add(self, numel, world, rank):
+        off = self.size
+        self.size += R.ratel_ssd_range_bytes(numel, world, rank)
+        return off
+
+    def open_direct(self):
+        import os
+        os.ftruncate(self.fd_buf, self.size)
+        os.fsync(self.fd_buf)
+        self.fd = os.open(self.path, os.O_RDWR | getattr(os, "O_DIRECT", 0))
+        return self.fd
+
+    def close(self):
+        import os
+        for fd in (self.fd, self.fd_buf):
+            if fd is not None:
+                os.close(fd)
+        self.fd = self.fd_buf = None
+
+
 class _Range:
-    def __init__(self, params, apply_wd, world, rank, dev, residency):
+    def __init__(self, params, apply_wd, world, rank, dev, residency, ssd=None):
         self.params = params
         self.numel = sum(p.numel() for p in params)
         cap = R.ratel_padded_numel(self.numel, world)
@@ -59,13 +91,23 @@ class _Range:
         self.g16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
         flat32 = torch.cat([p.detach().reshape(-1).to(torch.float32) for p in params]).to(dev)
         s = max(end - beg, 8)
-        if residency == "device":
-            mk = lambda: torch.zeros(s, dtype=torch.float32, device=dev)
+        self.ssd, self.ssd_off = ssd, None
+        if residency == "ssd":
+            # theta0 and zero moments go to the file; no state tensors are kept
+            import os
+            self.ssd_off = ssd.add(self.numel, world, rank)
+            self.ssd_stride = R.ratel_ssd_range_bytes(self.numel, world, rank) // 3
+            if end > beg:
+                os.pwrite(ssd.fd_buf, flat32[beg:end].cpu().numpy().tobytes(), self.ssd_off)
+            self.master = self.m = self.v = None
         else:
-            mk = lambda: torch.zeros(s, dtype=torch.float32).pin_memory()
-        self.master, self.m, self.v = mk(), mk(), mk()
-        if end > beg:
-            self.master[:end - beg].copy_(flat32[beg:end])
+            if residency == "device":
+                mk = lambda: torch.zeros(s, dtype=torch.float32, device=dev)
+            else:
+                mk = lambda: torch.zeros(s, dtype=torch.float32).pin_memory()
+            self.master, self.m, self.v = mk(), mk(), mk()
+            if end > beg:
+                self.master[:end - beg].copy_(flat32[beg:end])
         self.p16[:self.numel].copy_(flat32.to(torch.bfloat16))
         off = 0
         for p in params:  # parameters become views of the flat buffers
@@ -79,12 +121,39 @@ class _Range:
     def ratel_range(self):
         return R.make_range(self.p16, self.g16, self.master, self.m, self.v, self.numel, int(self.apply_wd))
 
+    def states(self):
+        """(master, exp_avg, exp_avg_sq) of this rank's slice as CPU/device
+        tensors (SSD: read back from the state file)."""
+        if self.ssd is None:
+            return self.master, self.m, self.v
+        import os
+        import numpy as np
+        n = self.slice[1] - self.slice[0]
+        rd = lambda k: torch.from_numpy(np.frombuffer(os.pread(self.ssd.fd_buf, 4 * n, self.ssd_off + k * self.ssd_stride),
+                                                      dtype=np.float32).copy())
+        return rd(0), rd(1), rd(2)
+
+    def load_states(self, master, m, v):
+        if self.ssd is None:
+            self.master.copy_(master)
+            self.m.copy_(m)
+            self.v.copy_(v)
+            return
+        import os
+        n = self.slice[1] - self.slice[0]
+        for k, t in enumerate((master, m, v)):
+            os.pwrite(self.ssd.fd_buf, t[:n].to(torch.float32).contiguous().numpy().tobytes(),
+                      self.ssd_off + k * self.ssd_stride)
+        os.fsync(self.ssd.fd_buf)
+
 
 class Ratel_Optimizer:
     """AdamW (or Adam-L2) over flat per-block buffers, driven by hand-offs.
 
-    residency: "device" (states in HBM), "host" (pinned host, GPU-streamed) or
-    "hostcompute" (pinned host, the paper's CPU handler).
+    residency: "device" (states in HBM), "host" (pinned host, GPU-streamed),
+    "hostcompute" (pinned host, the paper's CPU handler) or "ssd" (a state file
+    at `ssd_path`, streamed by the library's reader/writer threads; the paper's
+    storage tier, single rank).
 
     granularity: "block" hands a transformer block off when its last gradient
     has accumulated; "tensor" registers every weight matrix of a block as its
@@ -96,7 +165,7 @@ class Ratel_Optimizer:
     `blocks`/`block_ids`/`state(i)` then index units."""
 
     def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,
-                 residency="device", no_decay=None, first_block_id=0, granularity="block"):
+                 residency="device", no_decay=None, first_block_id=0, granularity="block", ssd_path=None):
         import torch.distributed as dist
         distributed = dist.is_available() and dist.is_initialized()
         world = dist.get_world_size() if distributed else 1
@@ -122,14 +191,22 @@ class Ratel_Optimizer:
                 units += [[([p], True)] for p in decay]
                 if nodecay:
                     units.append([(nodecay, False)])
+        if residency == "ssd" and not ssd_path:
+            raise ValueError('residency="ssd" needs ssd_path (the state file to create)')
+        self.ssd = _SsdFile(ssd_path) if residency == "ssd" else None
         for j, groups in enumerate(units):
-            ranges = [_Range(ps, wd, world, rank, dev, residency) for ps, wd in groups]
-            bid = first_block_id + j
+            ranges = [_Range(ps, wd, world, rank, dev, residency, self.ssd) for ps, wd in groups]
+            self.blocks.append(ranges)
+            self.block_ids.append(first_block_id + j)
+        if self.ssd is not None:
+            self.ssd.open_direct()
+        for bid, ranges in zip(self.block_ids, self.blocks):
             R.ratel_register_block(bid, [r.ratel_range() for r in ranges],
                                    {"device": R.RATEL_DEVICE, "host": R.RATEL_PINNED_HOST,
-                                    "hostcompute": R.RATEL_HOST_COMPUTE}[residency])
-            self.blocks.append(ranges)
-            self.block_ids.append(bid)
+                                    "hostcompute": R.RATEL_HOST_COMPUTE, "ssd": R.RATEL_SSD}[residency])
+            if self.ssd is not None:
+                for i, r in enumerate(ranges):
+                    R.ratel_register_ssd(bid, i, self.ssd.fd, r.ssd_off)
         self._pending = {}
         self._handed = set()
         self._hooks = []
@@ -182,10 +259,15 @@ class Ratel_Optimizer:
         """Step counter and copies of every range's fp32 master/exp_avg/
         exp_avg_sq (this rank's slices).  Call between steps."""
         torch.cuda.synchronize()
+        out = []
+        for ranges in self.blocks:
+            out.append([])
+            for r in ranges:
+                master, m, v = r.states()
+                out[-1].append({"master": master.detach().cpu().clone(), "exp_avg": m.detach().cpu().clone(),
+                                "exp_avg_sq": v.detach().cpu().clone()})
         return {"t": self.t, "lr": self.lr, "betas": self.betas, "eps": self.eps,
-                "weight_decay": self.weight_decay,
-                "ranges": [[{"master": r.master.detach().cpu().clone(), "exp_avg": r.m.detach().cpu().clone(),
-                             "exp_avg_sq": r.v.detach().cpu().clone()} for r in ranges] for ranges in self.blocks]}
+                "weight_decay": self.weight_decay, "ranges": out}
 
     def load_state_dict(self, sd: dict) -> None:
         """Restore states saved by state_dict() (same block/range layout) and
@@ -195,24 +277,28 @@ class Ratel_Optimizer:
         for ranges, saved in zip(self.blocks, sd["ranges"]):
             assert len(ranges) == len(saved)
             for r, s in zip(ranges, saved):
-                r.master.copy_(s["master"])
-                r.m.copy_(s["exp_avg"])
-                r.v.copy_(s["exp_avg_sq"])
+                r.load_states(s["master"], s["exp_avg"], s["exp_avg_sq"])
                 beg, end = r.slice
                 if end > beg:  # the model's working copy must match the restored master
-                    r.p16[beg:end].copy_(r.master[:end - beg].to(r.p16.device).to(torch.bfloat16))
+                    r.p16[beg:end].copy_(s["master"][:end - beg].to(r.p16.device).to(torch.bfloat16))
         self.t = int(sd["t"])
         self.lr, self.betas, self.eps, self.weight_decay = sd["lr"], tuple(sd["betas"]), sd["eps"], sd["weight_decay"]
         torch.cuda.synchronize()
 
     def state(self, block_index: int):
-        """(master, exp_avg, exp_avg_sq, p16, g16) flat views of each range of a block."""
-        return [(r.master, r.m, r.v, r.p16, r.g16) for r in self.blocks[block_index]]
+        """(master, exp_avg, exp_avg_sq, p16, g16) flat views of each range of a
+        block (SSD: the states are copies read back from the file)."""
+        return [(*r.states(), r.p16, r.g16) for r in self.blocks[block_index]]
 
     def remove_hooks(self):
         for h in self._hooks:
             h.remove()
         self._hooks.clear()
+
+    def close(self):
+        """Release the SSD state file (after ratel_finalize / Ratel_init exit)."""
+        if self.ssd is not None:
+            self.ssd.close()
 
 
 def Ratel_hook(optimizer: Ratel_Optimizer) -> Ratel_Optimizer:

@@ -140,3 +140,57 @@ def test_paper_api_tensor_granularity_bitwise(cuda_dev, residency):
     for a, b in zip(out["block"][0], out["tensor"][0]):
         assert torch.equal(a, b)
     assert out["block"][1] == out["tensor"][1]
+
+
+def test_paper_api_ssd_residency_bitwise(cuda_dev, tmp_path):
+    """residency="ssd": the wrapper writes theta0 into one state file, hands
+    the library an O_DIRECT fd, and every step streams the states through the
+    reader/writer threads -- same bits as device residency (R16), and
+    state_dict() reads the file back; load_state_dict() into a fresh SSD
+    optimizer then continues bitwise like an uninterrupted run."""
+    def build():
+        torch.manual_seed(3)
+        return torch.nn.Sequential(*[Block(64) for _ in range(2)]).to(cuda_dev)
+
+    x = torch.randn(32, 64, device=cuda_dev, dtype=torch.bfloat16)
+
+    def train(model, opt, n):
+        for _ in range(n):
+            opt.begin_step()
+            model(x).float().pow(2).mean().backward()
+            opt.end_step()
+        torch.cuda.synchronize()
+
+    def snap(model, opt):
+        sd = opt.state_dict()
+        return ([p.detach().view(torch.int16).cpu().clone() for p in model.parameters()],
+                [t.view(torch.int32) for rs in sd["ranges"] for r in rs for t in r.values()])
+
+    cfg = dict(tile_elems=4096)
+    with Ratel_init(**cfg):
+        m0 = build()
+        o0 = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in m0]))
+        train(m0, o0, 5)
+        want = snap(m0, o0)
+        o0.remove_hooks()
+    with Ratel_init(**cfg):
+        m1 = build()
+        o1 = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in m1], residency="ssd",
+                                        ssd_path=str(tmp_path / "a.bin")))
+        train(m1, o1, 3)
+        sd = o1.state_dict()
+        o1.remove_hooks()
+    o1.close()
+    with Ratel_init(**cfg):
+        m2 = build()
+        o2 = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in m2], residency="ssd",
+                                        ssd_path=str(tmp_path / "b.bin")))
+        o2.load_state_dict(sd)
+        train(m2, o2, 2)
+        got = snap(m2, o2)
+        o2.remove_hooks()
+    o2.close()
+    for a, b in zip(want[0], got[0]):
+        assert torch.equal(a, b)
+    for a, b in zip(want[1], got[1]):
+        assert torch.equal(a, b)
