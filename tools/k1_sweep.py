@@ -35,6 +35,30 @@ def build():
             print(name, path)
 
 
+TMA_GRID = [  # (consumer warps, stages, CTAs per SM, evict-first) -- dynamic tile scheduling
+    (16, 3, 1, 0), (8, 6, 1, 0), (8, 8, 1, 0), (12, 5, 1, 0), (8, 4, 2, 0), (16, 2, 2, 0), (4, 7, 2, 0),
+    (16, 4, 1, 1), (8, 8, 1, 1)]
+if os.environ.get("RATEL_TMA_GRID"):   # e.g. "8,6,1,0;8,7,1,0"
+    TMA_GRID = [tuple(int(x) for x in g.split(",")) for g in os.environ["RATEL_TMA_GRID"].split(";")]
+
+
+def build_tma():
+    """TMA K1 geometry variants (the default is 16 warps x 4 stages x 1 CTA/SM)."""
+    from paper_conf_icde_liaosyxcyww25_b200 import _build
+    os.makedirs(VDIR, exist_ok=True)
+    for f in glob.glob(os.path.join(VDIR, "libratel_*.so")):
+        os.remove(f)
+    jobs = []
+    for w, st, c, ef in TMA_GRID:
+        name = f"tma_w{w}s{st}c{c}" + ("_ef" if ef else "")
+        jobs.append((name, [f"RATEL_TMA_CONSUMER_WARPS={w}", f"RATEL_TMA_STAGES={st}",
+                            f"RATEL_TMA_CTAS_PER_SM={c}", f"RATEL_TMA_EVICT_FIRST={ef}"]))
+    with ThreadPoolExecutor(8) as ex:
+        for name, path in zip([j[0] for j in jobs], ex.map(
+                lambda j: _build.build(out=os.path.join(VDIR, f"libratel_{j[0]}.so"), defines=j[1]), jobs)):
+            print(name, path)
+
+
 def copy_gbs(torch):
     a = torch.empty(1 << 30, dtype=torch.bfloat16, device="cuda")
     b = torch.empty_like(a)
@@ -79,7 +103,7 @@ def check_variant(torch, R, L, base_out=None):
     return out
 
 
-def run(nblocks=8, steps=10, warmup=3, rounds=3):
+def run(nblocks=8, steps=10, warmup=3, rounds=int(os.environ.get("RATEL_SWEEP_ROUNDS", "3"))):
     import torch
     from paper_conf_icde_liaosyxcyww25_b200 import ratel as R
     dev = torch.device("cuda:0")
@@ -152,5 +176,7 @@ def run(nblocks=8, steps=10, warmup=3, rounds=3):
 if __name__ == "__main__":
     if sys.argv[1] == "build":
         build()
+    elif sys.argv[1] == "build_tma":
+        build_tma()
     else:
         run(int(sys.argv[2]) if len(sys.argv) > 2 else 8)
