@@ -4,6 +4,7 @@ Bounds: DESIGN.md R13 (tests/tolerance.py) at tol 1e-5 -- BASELINE.json's
 "max relative error 1e-5" and "bf16 within 1 ulp" read against the scale the
 oracle tracks.  Self-consistency claims (R16) are bitwise.
 """
+import math
 import numpy as np
 import pytest
 import torch
@@ -502,6 +503,111 @@ def test_range_beyond_2pow32_elements_sampled_vs_oracle(cuda_dev):
         check_range(got, ref, own_rne=oracle.bf16_rne, what="2^32+ range")
         assert np.array_equal(got["p16"], oracle.bf16_rne(got["p32"]))
     del th, m, v, p, g
+    torch.cuda.empty_cache()
+
+
+def test_fullsize_30b_blocks_clip_sampled_vs_oracle(cuda_dev):
+    """BASELINE configs[2] block shape (616,655,872 params, h = 7168) with the
+    global grad-norm clip (max_norm 1.0) in the bench's launch configuration:
+    that block plus a small ragged one, two steps, device-generated inputs.  The oracle's norm runs
+    over every element of both blocks (synth's grads, fp64 in index order) and
+    must agree with the library's K2/K3 sum; sampled elements vs the oracle
+    with that coefficient; P16 == bf16(P32) everywhere."""
+    h = 7168
+    ns = [12 * h * h + 13 * h, 1_000_003]     # a full block and a small ragged one share the norm
+    nblk = 2
+    idxs = [np.unique(np.concatenate([np.arange(0, 64), np.arange(n - 64, n),
+                                      np.random.default_rng(4).integers(0, n, 100_000)])).astype(np.uint64)
+            for n in ns]
+    state = []
+    with ratel_lib(max_grad_norm=1.0):
+        gs = [torch.empty(n, dtype=torch.bfloat16, device=cuda_dev) for n in ns]
+        for b in range(nblk):
+            n = ns[b]
+            th = torch.empty(n, dtype=torch.float32, device=cuda_dev)
+            R.ratel_gen_theta0(th.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, b))
+            m, v = torch.zeros(n, device=cuda_dev), torch.zeros(n, device=cuda_dev)
+            p = torch.zeros(n, dtype=torch.bfloat16, device=cuda_dev)
+            state.append((p, th, m, v))
+            R.ratel_register_block(b, [R.make_range(p, gs[b], th, m, v, n)], R.RATEL_DEVICE)
+        refs = [oracle.Range.fresh(synth.theta0_at(idxs[b], block=b)) for b in range(nblk)]
+        for t in (1, 2):
+            S, parts = 0.0, []
+            for b in range(nblk):
+                n = ns[b]
+                R.ratel_gen_grad16(gs[b].data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, b))
+                g16 = synth.grad16(n, step=t, block=b)
+                S = oracle.grad_sumsq(g16, S)
+                for c in range(0, n, 1 << 24):   # squares of bf16 values are exact in fp64; pairwise sums
+                    x = synth.bf16_bits_to_f32(g16[c:c + (1 << 24)]).astype(np.float64)
+                    parts.append(float(np.sum(x * x)))
+            S_acc = math.fsum(parts)             # accurate to ~1e-15 relative
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            for b in reversed(range(nblk)):
+                R.ratel_offload_grad_chunk(b, None)
+            R.ratel_sync(None)
+            s_gpu = R.ratel_get_grad_sumsq()
+            # the library's fp64 tree of per-CTA partials is accurate; the oracle's plain
+            # index-order recursion is within its textbook bound (n-1)*u*S (u = 2^-53)
+            assert abs(s_gpu - S_acc) <= 1e-12 * S_acc, (s_gpu, S_acc)
+            assert abs(S - S_acc) <= sum(ns) * 2.0 ** -53 * S_acc, (S, S_acc)
+            coef = oracle.clip_coef(S, 1.0)
+            assert coef < 1.0                     # the clip is active at this size
+            for b in range(nblk):
+                oracle.adam_range(refs[b], synth.grad16_at(idxs[b], step=t, block=b), oracle.hparams(step=t),
+                                  coef=coef)
+        for b in range(nblk):
+            ii = torch.from_numpy(idxs[b].astype(np.int64)).to(cuda_dev)
+            p, th, m, v = state[b]
+            got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
+                       p16=torch_to_u16(p[ii]))
+            check_range(got, refs[b], own_rne=oracle.bf16_rne, what=f"30B block {b} (clip)")
+            assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
+    del state, gs
+    torch.cuda.empty_cache()
+
+
+def test_fullsize_70b_block_pinned_host_sampled_vs_oracle(cuda_dev):
+    """BASELINE configs[3] block shape (805,412,864 params, h = 8192) with
+    theta/m/v in exact-size pinned host memory, streamed through the default
+    tile ring (the bench's host configuration): two steps, sampled elements vs
+    the oracle, P16 == bf16(P32) on every element."""
+    h = 8192
+    n = 12 * h * h + 13 * h
+    idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(n - 64, n),
+                                    np.random.default_rng(6).integers(0, n, 100_000)])).astype(np.uint64)
+    owners = [R.pinned_tensor(n) for _ in range(3)]
+    th, m, v = (o.tensor for o in owners)
+    chunk = 1 << 26
+    tmp = torch.empty(chunk, dtype=torch.float32, device=cuda_dev)
+    for beg in range(0, n, chunk):
+        k = min(chunk, n - beg)
+        R.ratel_gen_theta0(tmp.data_ptr(), k, beg, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, 0))
+        th[beg:beg + k].copy_(tmp[:k])
+    del tmp
+    m.zero_()
+    v.zero_()
+    with ratel_lib():
+        p = torch.zeros(n, dtype=torch.bfloat16, device=cuda_dev)
+        g = torch.empty(n, dtype=torch.bfloat16, device=cuda_dev)
+        R.ratel_register_block(0, [R.make_range(p, g, th, m, v, n)], R.RATEL_PINNED_HOST)
+        ref = oracle.Range.fresh(synth.theta0_at(idx, block=0))
+        for t in (1, 2):
+            R.ratel_gen_grad16(g.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, 0))
+            R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, t)
+            R.ratel_offload_grad_chunk(0, None)
+            R.ratel_sync(None)
+            oracle.adam_range(ref, synth.grad16_at(idx, step=t, block=0), oracle.hparams(step=t))
+        ii = torch.from_numpy(idx.astype(np.int64))
+        got = dict(p32=th[ii].numpy().copy(), m32=m[ii].numpy().copy(), v32=v[ii].numpy().copy(),
+                   p16=torch_to_u16(p[ii.to(cuda_dev)]))
+        check_range(got, ref, own_rne=oracle.bf16_rne, what="70B block (pinned host)")
+        for beg in range(0, n, chunk):     # no staleness on every element
+            k = min(chunk, n - beg)
+            assert torch.equal(p[beg:beg + k].view(torch.int16),
+                               th[beg:beg + k].to(cuda_dev).to(torch.bfloat16).view(torch.int16))
+        del p, g
+    del th, m, v, owners
     torch.cuda.empty_cache()
 
 
