@@ -567,12 +567,13 @@ def test_fullsize_30b_blocks_clip_sampled_vs_oracle(cuda_dev):
     torch.cuda.empty_cache()
 
 
-def test_fullsize_70b_block_pinned_host_sampled_vs_oracle(cuda_dev):
-    """BASELINE configs[3] block shape (805,412,864 params, h = 8192) with
-    theta/m/v in exact-size pinned host memory, streamed through the default
-    tile ring (the bench's host configuration): two steps, sampled elements vs
-    the oracle, P16 == bf16(P32) on every element."""
-    h = 8192
+@pytest.mark.parametrize("h", [8192, 12288])
+def test_fullsize_70b_block_pinned_host_sampled_vs_oracle(cuda_dev, h):
+    """BASELINE configs[3] / configs[4] block shapes (70B: 805,412,864 params,
+    h = 8192; 175B: 1,812,099,072 params, h = 12288) with theta/m/v in
+    exact-size pinned host memory, streamed through the default tile ring (the
+    bench's host configuration): two steps, sampled elements vs the oracle,
+    P16 == bf16(P32) on every element."""
     n = 12 * h * h + 13 * h
     idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(n - 64, n),
                                     np.random.default_rng(6).integers(0, n, 100_000)])).astype(np.uint64)
@@ -601,7 +602,7 @@ def test_fullsize_70b_block_pinned_host_sampled_vs_oracle(cuda_dev):
         ii = torch.from_numpy(idx.astype(np.int64))
         got = dict(p32=th[ii].numpy().copy(), m32=m[ii].numpy().copy(), v32=v[ii].numpy().copy(),
                    p16=torch_to_u16(p[ii.to(cuda_dev)]))
-        check_range(got, ref, own_rne=oracle.bf16_rne, what="70B block (pinned host)")
+        check_range(got, ref, own_rne=oracle.bf16_rne, what=f"h={h} block (pinned host)")
         for beg in range(0, n, chunk):     # no staleness on every element
             k = min(chunk, n - beg)
             assert torch.equal(p[beg:beg + k].view(torch.int16),
