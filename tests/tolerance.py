@@ -35,6 +35,14 @@ def _nan_ok(a, b):
     return ~an
 
 
+def _absdiff(a, b):
+    """|a - b| in float64, 0 where the values are equal (so matching
+    infinities compare as equal instead of producing inf - inf = NaN)."""
+    a, b = np.asarray(a, np.float64), np.asarray(b, np.float64)
+    with np.errstate(invalid="ignore"):
+        return np.where(a == b, 0.0, np.abs(a - b))
+
+
 def check_range(got: dict, ref, tol: float = TOL, own_rne=None, what: str = "") -> dict:
     """got: dict with p32, m32, v32 (float32) and p16 (uint16) from the GPU.
     ref: oracle.Range after the same steps (carries theta_bar and m_bar).
@@ -46,7 +54,7 @@ def check_range(got: dict, ref, tol: float = TOL, own_rne=None, what: str = "") 
     rep = {}
 
     ok = _nan_ok(th, th_r)
-    e_th = np.abs(th[ok].astype(np.float64) - th_r[ok])
+    e_th = _absdiff(th[ok], th_r[ok])
     lim = tol * tbar[ok]
     bad = e_th > lim
     assert not bad.any(), (f"{what} theta: {bad.sum()} elements out of bound; worst "
@@ -54,21 +62,21 @@ def check_range(got: dict, ref, tol: float = TOL, own_rne=None, what: str = "") 
     rep["theta_scaled"] = float((e_th / np.maximum(tbar[ok], 1e-300)).max(initial=0.0))
 
     ok = _nan_ok(m, m_r)
-    e_m = np.abs(m[ok].astype(np.float64) - m_r[ok])
+    e_m = _absdiff(m[ok], m_r[ok])
     bad = e_m > tol * mbar[ok]
     assert not bad.any(), (f"{what} m: {bad.sum()} elements out of bound; worst abs "
                            f"{e_m[bad].max():.3e}")
     rep["m_scaled"] = float((e_m / np.maximum(mbar[ok], 1e-300)).max(initial=0.0))
 
     ok = _nan_ok(v, v_r)
-    e_v = np.abs(v[ok].astype(np.float64) - v_r[ok])
+    e_v = _absdiff(v[ok], v_r[ok])
     bad = e_v > tol * np.abs(v_r[ok].astype(np.float64))
     assert not bad.any(), f"{what} v: {bad.sum()} elements out of bound"
     rep["v_rel"] = float((e_v / np.maximum(np.abs(v_r[ok].astype(np.float64)), 1e-300)).max(initial=0.0))
 
     pv, pv_r = bf16_to_f64(p), bf16_to_f64(p_r)
     ok = _nan_ok(pv, pv_r)
-    e_p = np.abs(pv[ok] - pv_r[ok])
+    e_p = _absdiff(pv[ok], pv_r[ok])
     bad = e_p > bf16_ulp_at(tbar[ok])
     assert not bad.any(), f"{what} p16: {bad.sum()} elements beyond 1 bf16 ulp at scale"
     rep["p16_ulps_at_scale"] = float((e_p / bf16_ulp_at(tbar[ok])).max(initial=0.0))
