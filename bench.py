@@ -923,9 +923,12 @@ def main():
             n = args.oracle_sample
             threads = host_threads()
             v, done, dt = oracle_sample_rate(n, 2, threads, min_seconds=8.0)
+            v1, done1, dt1 = oracle_sample_rate(n // 8, 2, 1, min_seconds=3.0)
             cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
                    "sample": f"{n:,} params (slice of block 0), {done} steps in {dt:.1f} s, "
-                             f"OpenMP {threads} threads"}
+                             f"OpenMP {threads} threads",
+                   "single_thread": {"value": v1, "unit": UNIT, "cores": 1,
+                                     "sample": f"{n // 8:,} params, {done1} steps in {dt1:.1f} s"}}
 
         if rank == 0:
             line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
