@@ -30,6 +30,7 @@ static const char* errs(CUresult r) {
 }
 
 int main() {
+  cuInit(0);
   cudaFree(0);
   CUdevice dev;
   cuDeviceGet(&dev, 0);
@@ -41,18 +42,32 @@ int main() {
 
   const int n = 1 << 20;
   const size_t bytes = n * sizeof(float);
+  // handle types to try: the create call rejects some on some systems
+  const CUmemAllocationHandleType kinds[3] = {CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, CU_MEM_HANDLE_TYPE_FABRIC,
+                                              CU_MEM_HANDLE_TYPE_NONE};
+  const char* kname[3] = {"posix_fd", "fabric", "none"};
   CUmulticastObjectProp prop = {};
-  prop.numDevices = 1;
-  prop.size = bytes;
-  prop.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
-  size_t gran = 0;
-  CUresult r = cuMulticastGetGranularity(&gran, &prop, CU_MULTICAST_GRANULARITY_RECOMMENDED);
-  printf(", \"granularity\": \"%s\", \"gran_bytes\": %zu", errs(r), gran);
-  if (r != CUDA_SUCCESS || gran == 0) { printf("}\n"); return 0; }
-  prop.size = ((bytes + gran - 1) / gran) * gran;
   CUmemGenericAllocationHandle mch;
-  r = cuMulticastCreate(&mch, &prop);
-  printf(", \"create\": \"%s\"", errs(r));
+  size_t gran = 0;
+  CUresult r = CUDA_ERROR_UNKNOWN;
+  int kind = -1;
+  for (int k = 0; k < 3 && r != CUDA_SUCCESS; ++k) {
+    prop = {};
+    prop.numDevices = 1;
+    prop.size = bytes;
+    prop.handleTypes = kinds[k];
+    size_t gmin = 0;
+    CUresult rg = cuMulticastGetGranularity(&gmin, &prop, CU_MULTICAST_GRANULARITY_MINIMUM);
+    cuMulticastGetGranularity(&gran, &prop, CU_MULTICAST_GRANULARITY_RECOMMENDED);
+    printf(", \"%s_granularity\": \"%s\", \"%s_gran_min\": %zu, \"%s_gran_rec\": %zu", kname[k], errs(rg), kname[k],
+           gmin, kname[k], gran);
+    if (rg != CUDA_SUCCESS || gmin == 0) continue;
+    gran = gmin;
+    prop.size = ((bytes + gran - 1) / gran) * gran;
+    r = cuMulticastCreate(&mch, &prop);
+    printf(", \"%s_create\": \"%s\"", kname[k], errs(r));
+    if (r == CUDA_SUCCESS) kind = k;
+  }
   if (r != CUDA_SUCCESS) { printf("}\n"); return 0; }
   r = cuMulticastAddDevice(mch, dev);
   printf(", \"add_device\": \"%s\"", errs(r));
@@ -62,7 +77,7 @@ int main() {
   ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
   ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
   ap.location.id = 0;
-  ap.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+  ap.requestedHandleTypes = kinds[kind];
   CUmemGenericAllocationHandle uh;
   r = cuMemCreate(&uh, prop.size, &ap, 0);
   printf(", \"mem_create\": \"%s\"", errs(r));
