@@ -68,7 +68,14 @@ int main() {
     printf(", \"%s_create\": \"%s\"", kname[k], errs(r));
     if (r == CUDA_SUCCESS) kind = k;
   }
-  if (r != CUDA_SUCCESS) { printf("}\n"); return 0; }
+  if (r != CUDA_SUCCESS) {   // does the create accept a 2-device object (a multi-GPU job's shape)?
+    prop.numDevices = 2;
+    prop.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+    prop.size = 2097152;
+    CUresult r2 = cuMulticastCreate(&mch, &prop);
+    printf(", \"create_2dev\": \"%s\"}\n", errs(r2));
+    return 0;
+  }
   r = cuMulticastAddDevice(mch, dev);
   printf(", \"add_device\": \"%s\"", errs(r));
   if (r != CUDA_SUCCESS) { printf("}\n"); return 0; }
