@@ -15,7 +15,10 @@ Printed: ONE JSON line on rank 0.
              pinned host memory streamed by the library's tile ring, grads
              H2D from pinned host and P16 D2H, all inside the timed region
   roofline   the update kernel K1: 28 algorithmic B/param / its event-timed
-             launch durations vs MEASURED_PEAKS.json hbm_gbs
+             launch durations vs MEASURED_PEAKS.json hbm_gbs (pinned-host
+             states: 24 B/param over the host link vs this run's duplex
+             probe; HOST_COMPUTE: 32 B/param of host DRAM vs this run's
+             host_stream probe -- K1's numbers then under roofline.k1)
   cpu_baseline  the CPU oracle on a bounded sample, on this host's cores
 `--impl reference` times the oracle as the reference arm.
 """
@@ -605,6 +608,48 @@ def run_e2e_device(args, R, torch, dev, model, sizes, order, t, world):
             "host_link_frac": achieved / link["duplex"], "host_link_probe": link}, tt[0]
 
 
+K1_NAME = {0: "adam_update_tma_kernel (K1)", 1: "adam_update_kernel (K1, LDG)", 2: "adam_update_kernel (K1, LDG_LITE)"}
+
+
+def host_dram_probe():
+    """Host DRAM ceiling for the CPU handler: tools/host_stream.c (OpenMP, all
+    cores) built with gcc into build/ and run; its 5-read/4-write pattern moves
+    the handler's 28 B/param."""
+    src = os.path.join(ROOT, "tools", "host_stream.c")
+    exe = os.path.join(ROOT, "build", "host_stream")
+    if not os.path.exists(exe) or os.path.getmtime(exe) < os.path.getmtime(src):
+        os.makedirs(os.path.dirname(exe), exist_ok=True)
+        subprocess.run(["gcc", "-O3", "-march=native", "-fopenmp", "-o", exe, src], check=True,
+                       capture_output=True)
+    out = subprocess.run([exe], check=True, capture_output=True, text=True, timeout=300).stdout
+    return json.loads(out.strip().splitlines()[-1])
+
+
+def offdevice_roofline(args, torch, dev, own_params_per_s, k1_roof):
+    """roofline for a step whose states live off the device:
+    pinned-host -- 12 B/param H2D + 12 B/param D2H of theta/m/v over the host
+    link vs the duplex probe of this run; HOST_COMPUTE -- the CPU handler's
+    28 B/param plus the 4 B/param of G16/P16 DMA through host DRAM vs the same
+    run's host_stream probe.  The tile kernel's HBM numbers stay under "k1"."""
+    k1 = {k: v for k, v in k1_roof.items() if k not in ("traffic", "ncu_dram_pct_of_peak")}
+    if args.residency == "host":
+        link = host_link_probe(torch, dev)
+        achieved = 24 * own_params_per_s / 1e9
+        return {"bound": "host_link", "kernel": "pinned-host tile ring (H2D theta/m/v, K1 on the tile, D2H)",
+                "achieved": achieved, "peak": link["duplex"], "unit": "GB/s", "frac": achieved / link["duplex"],
+                "traffic": None, "algorithmic_bytes_per_param": 24,
+                "peak_source": "this run's pinned H2D || D2H probe on two streams", "host_link_probe": link,
+                "k1": k1}
+    probe = host_dram_probe()
+    achieved = 32 * own_params_per_s / 1e9
+    return {"bound": "host_dram", "kernel": "CPU AdamW handler (HOST_COMPUTE) + G16/P16 DMA",
+            "achieved": achieved, "peak": probe["adam_pattern_gbs"], "unit": "GB/s",
+            "frac": achieved / probe["adam_pattern_gbs"], "traffic": None,
+            "algorithmic_bytes_per_param": 32,
+            "peak_source": f"this run's tools/host_stream.c 5-read/4-write pattern, {probe['threads']} threads",
+            "host_dram_probe": probe}
+
+
 def host_link_probe(torch, dev, nbytes=1 << 30, reps=3):
     """Measured duplex host-link bandwidth on this box (pinned H2D and D2H
     concurrently on two streams): the e2e roofline denominator."""
@@ -866,7 +911,7 @@ def main():
         achieved = k1_bytes / (k1_ms / 1e3) / 1e9 if k1_ms > 0 else None
         tpp = ncu_traffic_per_param()
         per_launch = own * args.steps / max(k1_n, 1)
-        roof = {"bound": "hbm", "kernel": "adam_update_tma_kernel (K1)", "achieved": achieved, "peak": peak,
+        roof = {"bound": "hbm", "kernel": K1_NAME.get(args.k1_kernel, "K1"), "achieved": achieved, "peak": peak,
                 "unit": "GB/s", "frac": (achieved / peak) if achieved else None,
                 "traffic": (tpp * per_launch) if tpp else None,
                 "algorithmic_bytes_per_launch": BYTES_PER_PARAM * per_launch,
@@ -909,6 +954,11 @@ def main():
             torch.cuda.empty_cache()
         if e2e is None:
             e2e = e2e_host
+        if args.residency != "device":      # the bound is off-device: report that roofline, K1 beside it
+            try:
+                roof = offdevice_roofline(args, torch, dev, own * args.steps / (ms / 1e3), roof)
+            except Exception as ex:  # report, do not hide
+                roof = dict(roof, offdevice_error=repr(ex)[:300])
 
         overlap_host = None
         if args.overlap_host_tokens > 0 and world == 1 and args.residency == "device":
