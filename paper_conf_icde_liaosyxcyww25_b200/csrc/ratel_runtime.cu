@@ -1298,12 +1298,12 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     const size_t need = (G.reg.size() + 1) * static_cast<size_t>(G.k2_grid);
     if (need > G.partial_cap) {
       const size_t cap = std::max(need, 2 * G.partial_cap);
+      // Partials are per-step scratch (every K2 writes its block's slots before
+      // K3 reads them), so the old contents are not carried over; cudaFree
+      // waits for any kernel of the previous step still reading them.
       double* p = nullptr;
       CK(cudaMalloc(&p, cap * sizeof(double)));
-      if (G.d_partials) {
-        CK(cudaMemcpy(p, G.d_partials, G.partial_cap * sizeof(double), cudaMemcpyDeviceToDevice));
-        CK(cudaFree(G.d_partials));
-      }
+      if (G.d_partials) CK(cudaFree(G.d_partials));
       G.d_partials = p;
       G.partial_cap = cap;
     }

@@ -1,6 +1,8 @@
 """Small AGO steps through the C ABI for compute-sanitizer (memcheck,
 racecheck, synccheck): C1-sized ragged blocks, a capped grid so every CTA
-cycles the TMA stage ring, clip mode, and a pinned-host block."""
+cycles the TMA stage ring, clip mode, a pinned-host block, the register-staged
+LDG / LDG_LITE kernels, a non-persistent grid (cta_tiles), zero-copy staging
+and the fused-reduction kernels (K1-RS, K2-RS) at world 1."""
 import os
 import sys
 
@@ -12,12 +14,15 @@ import paper_conf_icde_liaosyxcyww25_b200 as R  # noqa: E402
 from tests.harness import GpuBlock, ratel_lib  # noqa: E402
 
 
-def run(max_ctas, clip, pinned):
+def run(max_ctas, clip, pinned, rs_scale=None, **cfg):
     dev = torch.device("cuda:0")
     blocks = [GpuBlock(0, [789_760 + 3], dev, pinned=pinned), GpuBlock(1, [40_001, 17], dev)]
-    with ratel_lib(max_ctas=max_ctas, max_grad_norm=clip, tile_elems=65_536):
+    with ratel_lib(max_ctas=max_ctas, max_grad_norm=clip, tile_elems=65_536, **cfg):
         for b in blocks:
             b.register()
+            if rs_scale is not None:
+                for i in range(len(b.sizes)):
+                    R.ratel_register_peer_grads(b.id, i, [None], rs_scale)
         for t in (1, 2):
             for b in blocks:
                 b.load_grads(t)
@@ -32,4 +37,10 @@ if __name__ == "__main__":
     run(4, 0.0, False)
     run(0, 1.0, False)
     run(2, 0.0, True)
+    run(8, 0.0, False, k1_kernel=R.RATEL_UPDATE_LDG)
+    run(0, 1.0, False, k1_kernel=R.RATEL_UPDATE_LDG_LITE)
+    run(0, 0.0, False, cta_tiles=4)
+    run(16, 0.0, True, staging=R.RATEL_STAGING_ZERO_COPY)
+    run(0, 0.0, False, rs_scale=0.5)
+    run(4, 1.0, True, rs_scale=0.5)
     print("sanitize_run: done")
