@@ -47,6 +47,11 @@
  * released before ratel_finalize destroys that stream).  The library owns only what
  * it creates: streams, events, device tiles, reduction buffers, NCCL comm.
  *
+ * CUDA graphs: the step is not graph-capturable (the library tracks its tile
+ * scheduler, arming state and collectives per call on the host); a stream
+ * passed to ratel_offload_grad_chunk / ratel_block_wait / ratel_sync while it
+ * is being captured is refused with RATEL_EINVAL before anything is enqueued.
+ *
  * Errors: every int-returning call returns RATEL_OK (0) or a negative code.
  * RATEL_EINVAL / RATEL_ESTATE have no side effects.  A CUDA or NCCL failure
  * (including an asynchronous one detected later) is STICKY: every later call

@@ -1488,9 +1488,27 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
   return RATEL_OK;
 }
 
+// The step is not graph-capturable: the tile scheduler's counters, the arming
+// state and the NCCL/host work are tracked per call on the host, so a replayed
+// capture would run stale launches.  A caller stream under capture is refused
+// before anything is enqueued (RATEL_EINVAL, no side effects).
+static int check_not_capturing(void* stream, const char* fn) {
+  cudaStreamCaptureStatus st = cudaStreamCaptureStatusNone;
+  const cudaError_t e = cudaStreamIsCapturing(static_cast<cudaStream_t>(stream), &st);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return set_error(RATEL_EINVAL, "%s: cannot use the stream (%s)", fn, cudaGetErrorString(e));
+  }
+  if (st != cudaStreamCaptureStatusNone)
+    return set_error(RATEL_EINVAL, "%s: the stream is being captured into a CUDA graph; the AGO step is not "
+                                   "graph-capturable", fn);
+  return RATEL_OK;
+}
+
 int ratel_offload_grad_chunk(int block_id, void* stream) {
   Nvtx nv("ratel_offload_grad_chunk %d", block_id);
   RK(entry());
+  RK(check_not_capturing(stream, "ratel_offload_grad_chunk"));
   if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
     return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d is not registered", block_id);
   Block& B = G.blocks[block_id];
@@ -1527,6 +1545,7 @@ int ratel_offload_grad_chunk(int block_id, void* stream) {
 
 int ratel_block_wait(int block_id, void* stream) {
   RK(entry());
+  RK(check_not_capturing(stream, "ratel_block_wait"));
   if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
     return set_error(RATEL_ESTATE, "ratel_block_wait: block %d is not registered", block_id);
   const Block& B = G.blocks[block_id];
@@ -1549,6 +1568,7 @@ int ratel_block_wait(int block_id, void* stream) {
 int ratel_sync(void* stream) {
   Nvtx nv("ratel_sync");
   RK(entry());
+  if (stream != nullptr) RK(check_not_capturing(stream, "ratel_sync"));
   if (G.armed || G.n_handed > 0) {
     if (!G.armed) return set_error(RATEL_ESTATE, "ratel_sync: blocks handed off but no ratel_adam_step");
     if (G.n_handed != static_cast<int>(G.reg.size()))

@@ -885,3 +885,32 @@ def test_alloc_pinned_states(cuda_dev):
         else:                                   # CPU handler: within the R13 bounds
             check_range(got, ref[0].oracle[0], own_rne=oracle.bf16_rne)
         del owners
+
+
+def test_graph_capture_is_refused_without_side_effects(cuda_dev):
+    """A caller stream under CUDA-graph capture is refused (RATEL_EINVAL)
+    before anything is enqueued; the step then completes normally and matches
+    the oracle."""
+    b = GpuBlock(0, [50_003], cuda_dev)
+    with ratel_lib():
+        b.register()
+        gs = b.load_grads(1)
+        torch.cuda.synchronize()
+        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], 1)
+        s = torch.cuda.Stream(device=cuda_dev)
+        g = torch.cuda.CUDAGraph()
+        codes = []
+        with pytest.warns(UserWarning, match="empty"), torch.cuda.graph(g, stream=s):
+            for call in (lambda: R.ratel_offload_grad_chunk(0, s.cuda_stream),
+                         lambda: R.ratel_block_wait(0, s.cuda_stream),
+                         lambda: R.ratel_sync(s.cuda_stream)):
+                try:
+                    call()
+                    codes.append(0)
+                except R.RatelError as e:
+                    codes.append(e.code)
+        assert codes == [R.RATEL_EINVAL] * 3, codes
+        R.ratel_offload_grad_chunk(0, None)     # not handed off by the refused call
+        R.ratel_sync(None)
+    oracle.adam_step(b.oracle, gs, oracle.hparams(step=1, **HP))
+    check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne, what="after refused capture")
