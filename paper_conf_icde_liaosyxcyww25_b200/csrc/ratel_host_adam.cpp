@@ -1,6 +1,10 @@
 // ratel_host_adam.cpp -- the CPU handler of RATEL_HOST_COMPUTE (see
 // ratel_host_adam.h).  Runs inside a cudaLaunchHostFunc callback, so it must
-// not call the CUDA API; it parallelises with OpenMP over 64K-element chunks.
+// not call the CUDA API; it parallelises with OpenMP over 64K-element chunks,
+// scheduled dynamically: with one team thread per core, the host's other
+// threads (the caller, the CUDA driver) preempt some team thread, and a static
+// split then waits for it (4.53 -> 5.03-5.08 G params/s on the 16-core box,
+// profiles/r01_hostcompute_sweep.jsonl).
 #include "ratel_host_adam.h"
 
 #include <omp.h>
@@ -100,7 +104,7 @@ void chunk(const HostAdamArgs& a, uint64_t i0, uint64_t i1) {
 void host_adam_range(const HostAdamArgs& a, int threads) {
   const uint64_t nchunks = (a.n + kChunk - 1) / kChunk;
   const int nt = threads > 0 ? threads : omp_get_max_threads();
-#pragma omp parallel for schedule(static) num_threads(nt)
+#pragma omp parallel for schedule(dynamic, 1) num_threads(nt)
   for (int64_t c = 0; c < static_cast<int64_t>(nchunks); ++c) {
     const uint64_t i0 = static_cast<uint64_t>(c) * kChunk;
     const uint64_t i1 = i0 + kChunk < a.n ? i0 + kChunk : a.n;
