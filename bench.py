@@ -207,8 +207,9 @@ def workload_config(args, world):
     if args.blocks:
         sizes = sizes[:args.blocks]
     P = sum(sizes)
-    resid = {"host": "pinned-host", "hostcompute": "pinned-host, CPU handler (HOST_COMPUTE)"}.get(
-        args.residency, "device")
+    resid = {"host": "pinned-host", "hostcompute": "pinned-host, CPU handler (HOST_COMPUTE)",
+             "hybrid": f"pinned-host, {args.hybrid_gpu_frac:.2f} of each block GPU-streamed + the rest by the CPU "
+                       f"handler"}.get(args.residency, "device")
     name = {"13B": "13B", "30B": "30B", "70B": "70B (Table IV shape, 64.9B)", "175B": "175B",
             "c1": "C1 tiny block"}[shape]
     return {"workload": f"{name} GPT model states ({len(sizes)} blocks), {resid}-resident, AdamW, "
@@ -626,28 +627,41 @@ def host_dram_probe():
 
 
 def offdevice_roofline(args, torch, dev, own_params_per_s, k1_roof):
-    """roofline for a step whose states live off the device:
-    pinned-host -- 12 B/param H2D + 12 B/param D2H of theta/m/v over the host
-    link vs the duplex probe of this run; HOST_COMPUTE -- the CPU handler's
-    28 B/param plus the 4 B/param of G16/P16 DMA through host DRAM vs the same
-    run's host_stream probe.  The tile kernel's HBM numbers stay under "k1"."""
+    """roofline for a step whose states live off the device.
+    A fraction f of the params is GPU-streamed (pinned-host tile ring: 12 B/param
+    H2D + 12 B/param D2H over the host link, the same 24 B/param through host
+    DRAM by DMA), the rest goes to the CPU handler (HOST_COMPUTE: 28 B/param of
+    CPU traffic + 4 B/param of G16/P16 DMA in host DRAM, 4 B/param on the link);
+    f = 1 for --residency host, 0 for hostcompute.  Each resource's achieved
+    bytes are set against this run's probe of it (duplex link probe,
+    tools/host_stream.c); the bound is the one closer to its peak.  The tile
+    kernel's HBM numbers stay under "k1"."""
+    f = {"host": 1.0, "hostcompute": 0.0}.get(args.residency, args.hybrid_gpu_frac)
     k1 = {k: v for k, v in k1_roof.items() if k not in ("traffic", "ncu_dram_pct_of_peak")}
-    if args.residency == "host":
+    legs = {}
+    if f > 0:
         link = host_link_probe(torch, dev)
-        achieved = 24 * own_params_per_s / 1e9
-        return {"bound": "host_link", "kernel": "pinned-host tile ring (H2D theta/m/v, K1 on the tile, D2H)",
-                "achieved": achieved, "peak": link["duplex"], "unit": "GB/s", "frac": achieved / link["duplex"],
-                "traffic": None, "algorithmic_bytes_per_param": 24,
-                "peak_source": "this run's pinned H2D || D2H probe on two streams", "host_link_probe": link,
-                "k1": k1}
-    probe = host_dram_probe()
-    achieved = 32 * own_params_per_s / 1e9
-    return {"bound": "host_dram", "kernel": "CPU AdamW handler (HOST_COMPUTE) + G16/P16 DMA",
-            "achieved": achieved, "peak": probe["adam_pattern_gbs"], "unit": "GB/s",
-            "frac": achieved / probe["adam_pattern_gbs"], "traffic": None,
-            "algorithmic_bytes_per_param": 32,
-            "peak_source": f"this run's tools/host_stream.c 5-read/4-write pattern, {probe['threads']} threads",
-            "host_dram_probe": probe}
+        bpp = 24 * f + 4 * (1 - f)
+        a = bpp * own_params_per_s / 1e9
+        legs["host_link"] = {"achieved": a, "peak": link["duplex"], "frac": a / link["duplex"],
+                             "algorithmic_bytes_per_param": bpp, "probe": link,
+                             "peak_source": "this run's pinned H2D || D2H probe on two streams"}
+    if f < 1:
+        probe = host_dram_probe()
+        bpp = 24 * f + 32 * (1 - f)
+        a = bpp * own_params_per_s / 1e9
+        legs["host_dram"] = {"achieved": a, "peak": probe["adam_pattern_gbs"], "frac": a / probe["adam_pattern_gbs"],
+                             "algorithmic_bytes_per_param": bpp, "probe": probe,
+                             "peak_source": f"this run's tools/host_stream.c 5-read/4-write pattern, "
+                                            f"{probe['threads']} threads"}
+    bound = max(legs, key=lambda k: legs[k]["frac"])
+    b = legs[bound]
+    kernel = {1.0: "pinned-host tile ring (H2D theta/m/v, K1 on the tile, D2H)",
+              0.0: "CPU AdamW handler (HOST_COMPUTE) + G16/P16 DMA"}.get(
+        f, f"{f:.2f} pinned-host tile ring + {1 - f:.2f} CPU handler")
+    return {"bound": bound, "kernel": kernel, "achieved": b["achieved"], "peak": b["peak"], "unit": "GB/s",
+            "frac": b["frac"], "traffic": None, "algorithmic_bytes_per_param": b["algorithmic_bytes_per_param"],
+            "peak_source": b["peak_source"], **legs, "k1": k1}
 
 
 def host_link_probe(torch, dev, nbytes=1 << 30, reps=3):
@@ -774,7 +788,10 @@ def main():
     ap.add_argument("--impl", default="ratel", choices=["ratel", "reference"])
     ap.add_argument("--shape", default="13B", choices=list(SHAPES))
     ap.add_argument("--blocks", type=int, default=0, help="use only the first N blocks")
-    ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute"])
+    ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute", "hybrid"])
+    ap.add_argument("--hybrid-gpu-frac", type=float, default=0.3,
+                    help="hybrid residency: fraction of each block streamed through the GPU (pinned-host tile "
+                         "ring); the rest is updated by the CPU handler (HOST_COMPUTE)")
     ap.add_argument("--host-threads", type=int, default=0)
     ap.add_argument("--clip", type=float, default=0.0)
     ap.add_argument("--max-ctas", type=int, default=0)
@@ -862,12 +879,29 @@ def main():
         model = Model(R, torch, dev, sizes, world, rank, "device" if args.residency == "device" else "host",
                       symm=fused)
         res = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
+        hybrid = args.residency == "hybrid"
+        if hybrid and world > 1:
+            raise SystemExit("--residency hybrid is single-rank")
         for b in range(len(sizes)):
+            if hybrid:   # block b = GPU-streamed head (id b) + CPU-handler tail (id b + L), handed off together
+                r = model.ranges[b]
+                k = min(sizes[b], int(round(args.hybrid_gpu_frac * sizes[b] / 8)) * 8)
+                head = R.make_range(r.param_bf16, r.grad_bf16, r.master, r.exp_avg, r.exp_avg_sq, k)
+                tail = R.make_range(r.param_bf16 + 2 * k, r.grad_bf16 + 2 * k, r.master + 4 * k, r.exp_avg + 4 * k,
+                                    r.exp_avg_sq + 4 * k, sizes[b] - k)
+                if k > 0:
+                    R.ratel_register_block(b, [head], R.RATEL_PINNED_HOST)
+                if k < sizes[b]:
+                    R.ratel_register_block(b + len(sizes), [tail], R.RATEL_HOST_COMPUTE)
+                continue
             R.ratel_register_block(b, [model.ranges[b]], res)
             if fused:   # update kernel stores P16 into every peer over NVLink; no NCCL all-gather
                 R.ratel_register_peer_params(b, 0, model.peer_ptrs[b])
         s = torch.cuda.Stream(device=dev)
         order = list(reversed(range(len(sizes))))          # decreasing index
+        if hybrid:
+            order = [x for b in order for x, on in ((b, args.hybrid_gpu_frac > 0),
+                                                    (b + len(sizes), args.hybrid_gpu_frac < 1)) if on]
         t = 1
         for _ in range(args.warmup):
             step_once(R, t, order, s)

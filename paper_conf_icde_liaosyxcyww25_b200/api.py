@@ -121,6 +121,18 @@ class _Range:
     def ratel_range(self):
         return R.make_range(self.p16, self.g16, self.master, self.m, self.v, self.numel, int(self.apply_wd))
 
+    def split_ranges(self, frac):
+        """(head, tail) library ranges for the hybrid residency (single rank):
+        elements [0, k) and [k, numel), k = frac * numel rounded to a multiple
+        of 8 (16-byte alignment); None for an empty part."""
+        k = min(self.numel, max(0, int(round(frac * self.numel / 8)) * 8))
+        wd = int(self.apply_wd)
+        ptr = lambda t, off, size: t.data_ptr() + off * size
+        head = R.make_range(self.p16, self.g16, self.master, self.m, self.v, k, wd) if k > 0 else None
+        tail = (R.make_range(ptr(self.p16, k, 2), ptr(self.g16, k, 2), ptr(self.master, k, 4), ptr(self.m, k, 4),
+                             ptr(self.v, k, 4), self.numel - k, wd) if k < self.numel else None)
+        return head, tail
+
     def states(self):
         """(master, exp_avg, exp_avg_sq) of this rank's slice as CPU/device
         tensors (SSD: read back from the state file)."""
@@ -151,9 +163,12 @@ class Ratel_Optimizer:
     """AdamW (or Adam-L2) over flat per-block buffers, driven by hand-offs.
 
     residency: "device" (states in HBM), "host" (pinned host, GPU-streamed),
-    "hostcompute" (pinned host, the paper's CPU handler) or "ssd" (a state file
-    at `ssd_path`, streamed by the library's reader/writer threads; the paper's
-    storage tier, single rank).
+    "hostcompute" (pinned host, the paper's CPU handler), "hybrid" (pinned host;
+    the first `hybrid_gpu_frac` of every range GPU-streamed, the rest updated
+    by the CPU handler -- two library blocks per unit, handed off together, so
+    the host link and the host's cores work on one block at the same time;
+    single rank) or "ssd" (a state file at `ssd_path`, streamed by the
+    library's reader/writer threads; the paper's storage tier, single rank).
 
     granularity: "block" hands a transformer block off when its last gradient
     has accumulated; "tensor" registers every weight matrix of a block as its
@@ -165,7 +180,8 @@ class Ratel_Optimizer:
     `blocks`/`block_ids`/`state(i)` then index units."""
 
     def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,
-                 residency="device", no_decay=None, first_block_id=0, granularity="block", ssd_path=None):
+                 residency="device", no_decay=None, first_block_id=0, granularity="block", ssd_path=None,
+                 hybrid_gpu_frac=0.3):
         import torch.distributed as dist
         distributed = dist.is_available() and dist.is_initialized()
         world = dist.get_world_size() if distributed else 1
@@ -191,16 +207,33 @@ class Ratel_Optimizer:
                 units += [[([p], True)] for p in decay]
                 if nodecay:
                     units.append([(nodecay, False)])
+        if residency == "hybrid" and world > 1:
+            raise ValueError('residency="hybrid" is single-rank')
         if residency == "ssd" and not ssd_path:
             raise ValueError('residency="ssd" needs ssd_path (the state file to create)')
         self.ssd = _SsdFile(ssd_path) if residency == "ssd" else None
         for j, groups in enumerate(units):
-            ranges = [_Range(ps, wd, world, rank, dev, residency, self.ssd) for ps, wd in groups]
+            ranges = [_Range(ps, wd, world, rank, dev, "host" if residency == "hybrid" else residency, self.ssd)
+                      for ps, wd in groups]
             self.blocks.append(ranges)
             self.block_ids.append(first_block_id + j)
         if self.ssd is not None:
             self.ssd.open_direct()
+        self._lib_ids = {}   # unit id -> the library blocks handed off for it
         for bid, ranges in zip(self.block_ids, self.blocks):
+            if residency == "hybrid":
+                tail_id = bid + len(units)
+                head, tail = zip(*[r.split_ranges(hybrid_gpu_frac) for r in ranges])
+                head, tail = [x for x in head if x is not None], [x for x in tail if x is not None]
+                self._lib_ids[bid] = []
+                if head:
+                    R.ratel_register_block(bid, head, R.RATEL_PINNED_HOST)
+                    self._lib_ids[bid].append(bid)
+                if tail:
+                    R.ratel_register_block(tail_id, tail, R.RATEL_HOST_COMPUTE)
+                    self._lib_ids[bid].append(tail_id)
+                continue
+            self._lib_ids[bid] = [bid]
             R.ratel_register_block(bid, [r.ratel_range() for r in ranges],
                                    {"device": R.RATEL_DEVICE, "host": R.RATEL_PINNED_HOST,
                                     "hostcompute": R.RATEL_HOST_COMPUTE, "ssd": R.RATEL_SSD}[residency])
@@ -225,7 +258,8 @@ class Ratel_Optimizer:
             if left == 0 and bid not in self._handed:
                 self._handed.add(bid)
                 # the active message: gradient complete on the stream backward used
-                R.ratel_offload_grad_chunk(bid, torch.cuda.current_stream())
+                for lid in self._lib_ids[bid]:
+                    R.ratel_offload_grad_chunk(lid, torch.cuda.current_stream())
         return hook
 
     # ------------------------------------------------------------- a step
@@ -252,7 +286,8 @@ class Ratel_Optimizer:
         for bid in self.block_ids:
             if bid not in self._handed:
                 self._handed.add(bid)
-                R.ratel_offload_grad_chunk(bid, s)
+                for lid in self._lib_ids[bid]:
+                    R.ratel_offload_grad_chunk(lid, s)
         R.ratel_sync(s)
 
     def state_dict(self) -> dict:

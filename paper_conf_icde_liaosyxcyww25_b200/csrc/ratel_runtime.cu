@@ -80,7 +80,7 @@ struct Block {
   std::vector<ratel_range> ranges;
   std::vector<Slice> slices;
   cudaEvent_t ev_grad = nullptr;  // "gradient arrived" -- recorded on the caller's stream
-  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt (s_h2d for HOST_COMPUTE)
+  cudaEvent_t ev_done = nullptr;  // this rank's P16 slices written -- on s_opt (s_hc_h2d for HOST_COMPUTE)
   cudaEvent_t ev_gh = nullptr;    // HOST_COMPUTE: G16 slices landed in host staging
   cudaEvent_t ev_hc = nullptr;    // HOST_COMPUTE: the CPU update of this block finished (on s_host)
   std::vector<uint16_t*> h_g, h_p;  // HOST_COMPUTE: pinned G16 / P16 staging per range (rank slice)
@@ -154,11 +154,15 @@ struct Ctx {
   int sms = 0, k1_grid = 0, k2_grid = 0, rs_grid = 0, lite_grid = 0;
   cudaStream_t s_opt = nullptr, s_h2d = nullptr, s_d2h = nullptr, s_comm = nullptr, s_host = nullptr,
                s_tile = nullptr;
+  // HOST_COMPUTE's own copy streams (G16 down, P16 up): kept apart from the
+  // tile ring's s_h2d/s_d2h so CPU-handler blocks and GPU-streamed blocks in
+  // one step do not queue behind each other's copies.
+  cudaStream_t s_hc_d2h = nullptr, s_hc_h2d = nullptr;
   // Device-residency update kernels alternate over s_k[0..update_streams-1];
   // s_opt joins each (ev_done) so it stays ordered after every grad read.
   cudaStream_t s_k[2] = {nullptr, nullptr};
   unsigned k_next = 0;
-  static constexpr int kNS = 11;  // every stream (8 + the SSD engine's 3), for the sync cross-waits
+  static constexpr int kNS = 13;  // every stream (10 + the SSD engine's 3), for the sync cross-waits
   cudaEvent_t ev_end[kNS] = {};
   cudaEvent_t ev_norm = nullptr;  // clip: global norm final (on s_opt)
   double* h_sumsq = nullptr;      // clip + HOST_COMPUTE: pinned copy of the norm
@@ -574,7 +578,7 @@ void CUDART_CB host_adam_cb(void* arg) {
 // The paper-literal handler: G16 device->host, CPU AdamW on the host states,
 // P16 host->device -- all stream-ordered (cudaLaunchHostFunc), no host blocking.
 int enqueue_host_compute(Block& B) {
-  CK(cudaStreamWaitEvent(G.s_d2h, B.ev_grad, 0));
+  CK(cudaStreamWaitEvent(G.s_hc_d2h, B.ev_grad, 0));
   HostTask* task = new HostTask();
   task->threads = G.cfg.host_threads;
   if (G.cfg.max_grad_norm > 0.0) {
@@ -586,7 +590,7 @@ int enqueue_host_compute(Block& B) {
     const Slice& s = B.slices[i];
     const uint64_t n = s.end - s.begin;
     if (n == 0) continue;
-    if (cudaMemcpyAsync(B.h_g[i], grad_ptr(r, s), n * 2, cudaMemcpyDeviceToHost, G.s_d2h) != cudaSuccess) {
+    if (cudaMemcpyAsync(B.h_g[i], grad_ptr(r, s), n * 2, cudaMemcpyDeviceToHost, G.s_hc_d2h) != cudaSuccess) {
       delete task;
       return sticky_fail(RATEL_ECUDA, "G16 D2H failed: %s", cudaGetErrorString(cudaGetLastError()));
     }
@@ -609,25 +613,25 @@ int enqueue_host_compute(Block& B) {
     a.coef = 1.0;
     task->ranges.push_back(a);
   }
-  cudaError_t e = cudaEventRecord(B.ev_gh, G.s_d2h);
+  cudaError_t e = cudaEventRecord(B.ev_gh, G.s_hc_d2h);
   if (e == cudaSuccess) e = cudaStreamWaitEvent(G.s_host, B.ev_gh, 0);
   if (e == cudaSuccess) e = cudaLaunchHostFunc(G.s_host, host_adam_cb, task);
   if (e != cudaSuccess) {
     delete task;
     return sticky_fail(RATEL_ECUDA, "host handler enqueue failed: %s", cudaGetErrorString(e));
   }
-  // P16 host->device on the H2D stream, so the host stream goes straight on to
-  // the next block's CPU update while this block's P16 crosses the link.
+  // P16 host->device on its own copy stream, so the host stream goes straight
+  // on to the next block's CPU update while this block's P16 crosses the link.
   CK(cudaEventRecord(B.ev_hc, G.s_host));
-  CK(cudaStreamWaitEvent(G.s_h2d, B.ev_hc, 0));
+  CK(cudaStreamWaitEvent(G.s_hc_h2d, B.ev_hc, 0));
   for (size_t i = 0; i < B.ranges.size(); ++i) {
     const Slice& s = B.slices[i];
     const uint64_t n = s.end - s.begin;
     if (n == 0) continue;
     CK(cudaMemcpyAsync(static_cast<uint16_t*>(B.ranges[i].param_bf16) + s.begin, B.h_p[i], n * 2,
-                       cudaMemcpyHostToDevice, G.s_h2d));
+                       cudaMemcpyHostToDevice, G.s_hc_h2d));
   }
-  CK(cudaEventRecord(B.ev_done, G.s_h2d));
+  CK(cudaEventRecord(B.ev_done, G.s_hc_h2d));
   return RATEL_OK;
 }
 
@@ -1083,7 +1087,8 @@ void destroy_all() {
   if (G.h_sumsq) cudaFreeHost(G.h_sumsq);
   if (G.ev_norm) cudaEventDestroy(G.ev_norm);
   if (G.comm) g_nccl.CommDestroy(G.comm);
-  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1],
+                         G.s_hc_d2h, G.s_hc_h2d})
     if (s) cudaStreamDestroy(s);
   G.~Ctx();
   new (&G) Ctx();
@@ -1111,6 +1116,8 @@ int init_body(int device, int rank, int world_size, const void* nccl_unique_id, 
   CK(cudaStreamCreateWithPriority(&G.s_comm, cudaStreamNonBlocking, greatest));
   CK(cudaStreamCreateWithPriority(&G.s_host, cudaStreamNonBlocking, greatest));
   CK(cudaStreamCreateWithPriority(&G.s_tile, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_hc_d2h, cudaStreamNonBlocking, greatest));
+  CK(cudaStreamCreateWithPriority(&G.s_hc_h2d, cudaStreamNonBlocking, greatest));
   CK(cudaEventCreateWithFlags(&G.ev_norm, cudaEventDisableTiming));
   for (cudaEvent_t& ev : G.ev_end) CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
   for (int k = 0; k < kMaxDepth; ++k) {
@@ -1479,7 +1486,7 @@ int ratel_adam_step(double lr, double beta1, double beta2, double eps, double we
   // the whole backward -- every handler stream waits for every gradient
   // handed off so far before any state moves (s_opt already waited on each).
   if (!G.pending.empty())
-    for (cudaStream_t st : {G.s_h2d, G.s_d2h, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
+    for (cudaStream_t st : {G.s_h2d, G.s_d2h, G.s_host, G.s_tile, G.s_k[0], G.s_k[1], G.s_hc_d2h, G.s_hc_h2d})
       for (int id : G.pending) CK(cudaStreamWaitEvent(st, G.blocks[id].ev_grad, 0));
   std::vector<cudaEvent_t> all_grads;  // SSD: no state is read before the whole backward
   for (int id : G.pending) all_grads.push_back(G.blocks[id].ev_grad);
@@ -1590,6 +1597,7 @@ int ratel_sync(void* stream) {
   RK(ssd_drain(true));
   const int NS = G.ssd != nullptr ? Ctx::kNS : Ctx::kNS - 3;
   cudaStream_t ss[Ctx::kNS] = {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1],
+                               G.s_hc_d2h, G.s_hc_h2d,
                                G.ssd ? G.ssd->s_in : nullptr, G.ssd ? G.ssd->s_k : nullptr,
                                G.ssd ? G.ssd->s_out : nullptr};
   for (int i = 0; i < NS; ++i) CK(cudaEventRecord(G.ev_end[i], ss[i]));
@@ -1622,7 +1630,8 @@ int ratel_sync(void* stream) {
 int ratel_finalize(void) {
   if (!G.inited) return set_error(RATEL_ESTATE, "ratel_finalize: not initialised");
   cudaSetDevice(G.device);
-  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1]})
+  for (cudaStream_t s : {G.s_opt, G.s_h2d, G.s_d2h, G.s_comm, G.s_host, G.s_tile, G.s_k[0], G.s_k[1],
+                         G.s_hc_d2h, G.s_hc_h2d})
     if (s) cudaStreamSynchronize(s);
   destroy_all();
   cudaGetLastError();
