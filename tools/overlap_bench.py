@@ -51,6 +51,7 @@ def run(args):
     R.ratel_finalize()
     ring = model.grad_ring
     res_code = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
+    hybrid = args.residency == "hybrid"
     vocab = bench.VOCAB if len(sizes) == L + 1 else 0
     hi = torch.cuda.Stream(priority=args.bwd_priority)
     order = list(reversed(range(len(sizes))))
@@ -72,16 +73,39 @@ def run(args):
         units[b] = [R.ratel_range(r0.param_bf16 + 2 * o, r0.grad_bf16 + 2 * o, 0, r0.master + 4 * o,
                                   r0.exp_avg + 4 * o, r0.exp_avg_sq + 4 * o, ln, 1) for (o, ln) in offs]
 
-    def uid(b, j):
-        return b * K + j
+    # Registered library blocks per unit: one, or with --residency hybrid the
+    # unit's first hybrid_gpu_frac GPU-streamed (PINNED_HOST) and the rest on
+    # the CPU handler (HOST_COMPUTE), handed off together.
+    lib = {}
+    nxt = 0
+    for b in range(len(sizes)):
+        for j, r in enumerate(units[b]):
+            parts = [(r, res_code)]
+            if hybrid:
+                k = min(r.numel, int(round(args.hybrid_gpu_frac * r.numel / 8)) * 8)
+                tail = R.ratel_range(r.param_bf16 + 2 * k, r.grad_bf16 + 2 * k, 0, r.master + 4 * k,
+                                     r.exp_avg + 4 * k, r.exp_avg_sq + 4 * k, r.numel - k, r.apply_weight_decay)
+                head = R.ratel_range(r.param_bf16, r.grad_bf16, 0, r.master, r.exp_avg, r.exp_avg_sq, k,
+                                     r.apply_weight_decay)
+                parts = [(x, c) for x, c, n in ((head, R.RATEL_PINNED_HOST, k),
+                                                (tail, R.RATEL_HOST_COMPUTE, r.numel - k)) if n > 0]
+            lib[(b, j)] = []
+            for x, c in parts:
+                lib[(b, j)].append((nxt, x, c))
+                nxt += 1
+
+    def handoff_unit(b, j, stream):
+        for i, _, _ in lib[(b, j)]:
+            R.ratel_offload_grad_chunk(i, stream)
 
     def handoff_all(b, stream):
         for j in range(len(units[b])):
-            R.ratel_offload_grad_chunk(uid(b, j), stream)
+            handoff_unit(b, j, stream)
 
     def wait_all(b, stream):
         for j in range(len(units[b])):
-            R.ratel_block_wait(uid(b, j), stream)
+            for i, _, _ in lib[(b, j)]:
+                R.ratel_block_wait(i, stream)
     t_state = {"t": 1}
 
     def arm():
@@ -111,10 +135,10 @@ def run(args):
                     if schedule != "deferred" and j >= args.ring:
                         wait_all(b + args.ring, hi)             # ring slot free
                     if len(units[b]) > 1:                       # per-tensor hand-off
-                        bw.block(b, b % args.ring, on_linear=lambda k, b=b: R.ratel_offload_grad_chunk(uid(b, k), hi))
+                        bw.block(b, b % args.ring, on_linear=lambda k, b=b: handoff_unit(b, k, hi))
                     else:
                         bw.block(b, b % args.ring)
-                        R.ratel_offload_grad_chunk(uid(b, 0), hi)
+                        handoff_unit(b, 0, hi)
                     if timeline:
                         tl["g"][b] = torch.cuda.Event(enable_timing=True)
                         tl["g"][b].record(hi)
@@ -137,9 +161,9 @@ def run(args):
             cfg.tile_elems = args.tile_elems
         cfg.staging = staging
         R.ratel_init(0, 0, 1, None, cfg)
-        for b in range(len(sizes)):
-            for j, r in enumerate(units[b]):
-                R.ratel_register_block(uid(b, j), [r], res_code)
+        for parts in lib.values():
+            for i, x, c in parts:
+                R.ratel_register_block(i, [x], c)
         t_state["t"] = 1
 
     for tokens in args.tokens:
@@ -184,7 +208,7 @@ def run(args):
                               clk.get("power_w"))
                 R.ratel_finalize()
             tb = times["bwd"][0]
-            row = {"residency": args.residency, "granularity": args.granularity, "cta_tiles": args.cta_tiles,
+            row = {"residency": args.residency + (f" {args.hybrid_gpu_frac}" if hybrid else ""), "granularity": args.granularity, "cta_tiles": args.cta_tiles,
                    "k1_kernel": args.k1_kernel, "bwd_priority": args.bwd_priority, "ring": args.ring,
                    "tile_elems": args.tile_elems, "zero_copy": bool(args.zero_copy),
                    "tokens": tokens, "max_ctas": mc,
@@ -211,7 +235,9 @@ if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("--shape", default="13B")
     ap.add_argument("--blocks", type=int, default=0)
-    ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute"])
+    ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute", "hybrid"])
+    ap.add_argument("--hybrid-gpu-frac", type=float, default=0.3,
+                    help="hybrid: fraction of each unit GPU-streamed; the rest goes to the CPU handler")
     ap.add_argument("--tokens", type=int, nargs="+", default=[2048, 8192, 32768])
     ap.add_argument("--max-ctas", type=int, nargs="+", default=[0, 32])
     ap.add_argument("--schedules", nargs="+", default=["bwd", "opt", "ago", "deferred", "naive"])
