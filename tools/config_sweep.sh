@@ -14,4 +14,8 @@ run --shape 70B --residency host --blocks 3 --steps 3 --warmup 3
 run --shape 175B --residency host --blocks 2 --steps 3 --warmup 3
 run --shape 13B --residency hostcompute --blocks 8 --steps 3 --warmup 3
 run --shape c1 --steps 200 --warmup 10
+
+# the hybrid residency (30 % GPU-streamed + 70 % CPU handler) on the C4 / C5 shapes
+run --shape 70B --residency hybrid --blocks 3 --steps 3 --warmup 3
+run --shape 175B --residency hybrid --blocks 2 --steps 3 --warmup 3
 echo done
