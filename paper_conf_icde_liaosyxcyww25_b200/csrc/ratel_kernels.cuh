@@ -721,6 +721,210 @@ __global__ void __launch_bounds__(kThreads, RATEL_K1_MINB) adam_update_rs_kernel
   if (P.any_peers) __threadfence_system();
 }
 
+// ---- K1-RS, TMA-staged variant (default with cfg.k1_kernel = TMA) ----------
+// The fused reduction with K1's data movement: a producer warp bulk-copies,
+// per 2048-element tile, every rank's G16 (the peers' through their P2P
+// mappings -- TMA keeps a stage's worth of NVLink reads in flight per SM
+// instead of a few registers' worth) plus theta, m, v into a shared-memory
+// ring of ~224 KB (8 stages at N = 1 down to 4 at N = 8); 8 consumer warps reduce the N gradients of their octet
+// in fp64 in rank order (reduce_g8's arithmetic, so the result is bitwise the
+// LDG kernel's), update, write theta/m/v and P16 back into the stage, and one
+// thread bulk-stores them (K1's release protocol 4).  Stage layout for nmax
+// = the largest rank count among the launch's ranges:
+//   [G16 rank 0 .. rank nmax-1 : 2 B x tile each][theta][m][v : 4 B x tile]
+// P16 is written over rank 0's G16 octet by the thread that read it.
+constexpr int kRsTmaConsumerWarps = 8;
+constexpr int kRsTmaThreads = 32 * (kRsTmaConsumerWarps + 1);
+constexpr int kRsTmaTile = kRsTmaConsumerWarps * 32 * 8;   // 2048 elements, one octet per consumer thread
+constexpr int kRsTmaMaxStages = 8;
+constexpr uint32_t kRsTmaRingBytes = 224 * 1024;           // the ring K1 keeps in flight per SM
+__host__ __device__ constexpr uint32_t rs_tma_stage_bytes(int nmax) {
+  return static_cast<uint32_t>(kRsTmaTile) * (2u * static_cast<uint32_t>(nmax) + 12u);
+}
+// As many stages as fill the ring (8 at N = 1, 4 at N = 8): bytes in flight
+// per SM stay at K1's level whatever the rank count.
+__host__ __device__ constexpr int rs_tma_stages(int nmax) {
+  return kRsTmaRingBytes / rs_tma_stage_bytes(nmax) < kRsTmaMaxStages
+             ? static_cast<int>(kRsTmaRingBytes / rs_tma_stage_bytes(nmax)) : kRsTmaMaxStages;
+}
+__host__ __device__ constexpr uint32_t rs_tma_smem_bytes(int nmax) {
+  return rs_tma_stages(nmax) * rs_tma_stage_bytes(nmax) + 3 * kRsTmaMaxStages * 8;
+}
+static_assert(rs_tma_smem_bytes(1) <= 227 * 1024 && rs_tma_smem_bytes(kMaxRanks) <= 227 * 1024,
+              "K1-RS TMA ring must fit the opt-in shared memory");
+
+__device__ __forceinline__ TileLoc locate_rs_tma_tile(const UpdateParams& P, uint64_t k) {
+  TileLoc t{0, 0, 0};
+  for (int r = 0; r < P.nr; ++r) {
+    const uint64_t body = P.r[r].n & ~7ull;
+    const uint64_t nt = (body + kRsTmaTile - 1) / kRsTmaTile;
+    if (k < nt) {
+      t.r = r;
+      t.off = k * kRsTmaTile;
+      t.len = static_cast<uint32_t>(body - t.off < (uint64_t)kRsTmaTile ? body - t.off : kRsTmaTile);
+      return t;
+    }
+    k -= nt;
+  }
+  t.r = -1;
+  return t;
+}
+
+template <int MODE, bool CLIP>
+__global__ void __launch_bounds__(kRsTmaThreads, 1) adam_update_rs_tma_kernel(const __grid_constant__ RsUpdateParams Q) {
+  const UpdateParams& P = Q.u;
+  extern __shared__ __align__(128) uint8_t smem[];
+  int nmax = 1;
+  for (int r = 0; r < P.nr; ++r) nmax = Q.gp[r].n > nmax ? Q.gp[r].n : nmax;
+  const uint32_t SB = rs_tma_stage_bytes(nmax);
+  const int NST = rs_tma_stages(nmax);
+  const uint32_t TH = static_cast<uint32_t>(nmax) * kRsTmaTile * 2u;  // theta's offset in a stage
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + NST * SB);
+  uint64_t* empty = full + kRsTmaMaxStages;
+  volatile uint64_t* tile_id = empty + kRsTmaMaxStages;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (threadIdx.x == 0) {
+    for (int st = 0; st < NST; ++st) {
+      mbar_init(&full[st], 1);
+      mbar_init(&empty[st], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  __syncthreads();
+  uint64_t total = 0;
+  for (int r = 0; r < P.nr; ++r) total += ((P.r[r].n & ~7ull) + kRsTmaTile - 1) / kRsTmaTile;
+
+  if (warp == kRsTmaConsumerWarps) {  // producer
+    if (lane == 0) {
+      const bool dyn = P.tile_ctr != nullptr;
+      uint64_t k = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : blockIdx.x;
+      int stage = 0;
+      uint32_t phase = 0;
+      for (;;) {
+        uint64_t kn = k;
+        if (k < total) kn = dyn ? atomicAdd(P.tile_ctr, 1ull) - P.tile_base : k + gridDim.x;
+        mbar_wait(&empty[stage], phase ^ 1);
+        if (k >= total) {
+          tile_id[stage] = ~0ull;
+          mbar_arrive(&full[stage]);
+          break;
+        }
+        tile_id[stage] = k;
+        const TileLoc t = locate_rs_tma_tile(P, k);
+        const RangeDesc& R = P.r[t.r];
+        const GradPeers& gp = Q.gp[t.r];
+        uint8_t* base = smem + stage * SB;
+        mbar_expect_tx(&full[stage], t.len * (2u * static_cast<uint32_t>(gp.n) + 12u));
+        for (int q = 0; q < gp.n; ++q) bulk_load(base + q * kRsTmaTile * 2, gp.g[q] + t.off, t.len * 2u, &full[stage]);
+        bulk_load(base + TH, R.th + t.off, t.len * 4u, &full[stage]);
+        bulk_load(base + TH + kRsTmaTile * 4, R.m + t.off, t.len * 4u, &full[stage]);
+        bulk_load(base + TH + kRsTmaTile * 8, R.v + t.off, t.len * 4u, &full[stage]);
+        if (++stage == NST) {
+          stage = 0;
+          phase ^= 1;
+        }
+        k = kn;
+      }
+    }
+  } else {  // consumers
+    const double coef_d = CLIP ? clip_coef_from(P.sumsq, P.max_norm, P.nonfinite_flag) : 1.0;
+    const float coef_f = static_cast<float>(coef_d);
+    int stage = 0, prev_stage = -1;
+    uint32_t phase = 0;
+    const uint32_t o = threadIdx.x;  // octet within the tile
+    for (;;) {
+      mbar_wait(&full[stage], phase);
+      const uint64_t k = tile_id[stage];
+      if (k == ~0ull) break;
+      const TileLoc t = locate_rs_tma_tile(P, k);
+      const RangeDesc& R = P.r[t.r];
+      const GradPeers& gp = Q.gp[t.r];
+      uint8_t* base = smem + stage * SB;
+      if (8 * o < t.len) {
+        uint4 w[kMaxRanks];
+#pragma unroll
+        for (int q = 0; q < kMaxRanks; ++q)
+          if (q < gp.n) w[q] = *reinterpret_cast<const uint4*>(base + q * kRsTmaTile * 2 + 16 * o);
+        double sd[8];
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk) sd[kk] = 0.0;
+#pragma unroll
+        for (int q = 0; q < kMaxRanks; ++q) {
+          if (q < gp.n) {
+            const uint32_t ws[4] = {w[q].x, w[q].y, w[q].z, w[q].w};
+#pragma unroll
+            for (int kk = 0; kk < 4; ++kk) {
+              sd[2 * kk] = __dadd_rn(sd[2 * kk], static_cast<double>(bf16_bits_to_f32(ws[kk] & 0xFFFFu)));
+              sd[2 * kk + 1] = __dadd_rn(sd[2 * kk + 1], static_cast<double>(bf16_bits_to_f32(ws[kk] >> 16)));
+            }
+          }
+        }
+        float4* th = reinterpret_cast<float4*>(base + TH) + 2 * o;
+        float4* mm = reinterpret_cast<float4*>(base + TH + kRsTmaTile * 4) + 2 * o;
+        float4* vv = reinterpret_cast<float4*>(base + TH + kRsTmaTile * 8) + 2 * o;
+        const float4 t0 = th[0], t1 = th[1], m0 = mm[0], m1 = mm[1], v0 = vv[0], v1 = vv[1];
+        float ft[8] = {t0.x, t0.y, t0.z, t0.w, t1.x, t1.y, t1.z, t1.w};
+        float fm[8] = {m0.x, m0.y, m0.z, m0.w, m1.x, m1.y, m1.z, m1.w};
+        float fv[8] = {v0.x, v0.y, v0.z, v0.w, v1.x, v1.y, v1.z, v1.w};
+        const bool wd = R.wd_on != 0;
+#pragma unroll
+        for (int kk = 0; kk < 8; ++kk)
+          adam_update<MODE, CLIP>(__double2float_rn(__dmul_rn(sd[kk], gp.scale)), ft[kk], fm[kk], fv[kk], P.s, wd,
+                                  coef_f, coef_d);
+        th[0] = make_float4(ft[0], ft[1], ft[2], ft[3]);
+        th[1] = make_float4(ft[4], ft[5], ft[6], ft[7]);
+        mm[0] = make_float4(fm[0], fm[1], fm[2], fm[3]);
+        mm[1] = make_float4(fm[4], fm[5], fm[6], fm[7]);
+        vv[0] = make_float4(fv[0], fv[1], fv[2], fv[3]);
+        vv[1] = make_float4(fv[4], fv[5], fv[6], fv[7]);
+        uint4 pk;
+        pk.x = pack_bf16x2_rn(ft[0], ft[1]);
+        pk.y = pack_bf16x2_rn(ft[2], ft[3]);
+        pk.z = pack_bf16x2_rn(ft[4], ft[5]);
+        pk.w = pack_bf16x2_rn(ft[6], ft[7]);
+        *reinterpret_cast<uint4*>(base + 16 * o) = pk;   // over rank 0's G16 octet (read above by this thread)
+        st_peers8(P.peers[t.r], t.off + 8 * o, pk);     // fused all-gather: NVLink P2P stores
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+      asm volatile("bar.sync 1, %0;" ::"r"(kRsTmaConsumerWarps * 32) : "memory");
+      if (threadIdx.x == 0) {
+        bulk_store(R.th + t.off, base + TH, t.len * 4u);
+        bulk_store(R.m + t.off, base + TH + kRsTmaTile * 4, t.len * 4u);
+        bulk_store(R.v + t.off, base + TH + kRsTmaTile * 8, t.len * 4u);
+        bulk_store(R.p + t.off, base, t.len * 2u);
+        asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        if (prev_stage >= 0) mbar_arrive(&empty[prev_stage]);
+        prev_stage = stage;
+      }
+      if (++stage == NST) {
+        stage = 0;
+        phase ^= 1;
+      }
+    }
+    if (threadIdx.x == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+    // scalar tails (< 8 elements per range), CTA 0
+    for (int r = 0; r < P.nr && blockIdx.x == 0; ++r) {
+      const RangeDesc& R = P.r[r];
+      const GradPeers& gp = Q.gp[r];
+      const uint64_t j = (R.n & ~7ull) + threadIdx.x;
+      if (j < R.n) {
+        float th = R.th[j], m = R.m[j], v = R.v[j];
+        adam_update<MODE, CLIP>(reduce_g1(gp, j), th, m, v, P.s, R.wd_on != 0, coef_f, coef_d);
+        R.th[j] = th;
+        R.m[j] = m;
+        R.v[j] = v;
+        const uint16_t pb = static_cast<uint16_t>(pack_bf16x2_rn(th, 0.0f) & 0xFFFFu);
+        R.p[j] = pb;
+        const PeerDesc& pd = P.peers[r];
+        for (int q = 0; q < pd.n; ++q) pd.p[q][j] = pb;
+      }
+    }
+    if (P.any_peers) __threadfence_system();
+  }
+}
+
 __device__ __forceinline__ double warp_sum(double x) {
 #pragma unroll
   for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);

@@ -319,6 +319,11 @@ void launch_k1(UpdateParams& P, unsigned grid, cudaStream_t st, int kernel) {
 template <int MODE, bool CLIP>
 cudaError_t prepare_k1() {
 #if RATEL_K1_TMA
+  const cudaError_t e = cudaFuncSetAttribute(adam_update_rs_tma_kernel<MODE, CLIP>,
+                                             cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             static_cast<int>(std::max(rs_tma_smem_bytes(1),
+                                                                       rs_tma_smem_bytes(kMaxRanks))));
+  if (e != cudaSuccess) return e;
   return cudaFuncSetAttribute(adam_update_tma_kernel<MODE, CLIP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                               static_cast<int>(kTmaSmemBytes));
 #else
@@ -329,6 +334,27 @@ cudaError_t prepare_k1() {
 template <int MODE, bool CLIP>
 void launch_k1_rs(RsUpdateParams& Q, unsigned grid, cudaStream_t st) {
   (void)grid;
+#if RATEL_K1_TMA
+  if (G.cfg.k1_kernel == RATEL_UPDATE_TMA) {  // TMA-staged fused reduction (one CTA per SM, persistent)
+    uint64_t tiles = 0;
+    int nmax = 1;
+    for (int r = 0; r < Q.u.nr; ++r) {
+      tiles += ((Q.u.r[r].n & ~7ull) + kRsTmaTile - 1) / kRsTmaTile;
+      nmax = std::max(nmax, Q.gp[r].n);
+    }
+    uint64_t cap = static_cast<uint64_t>(G.sms);
+    if (G.cfg.max_ctas > 0) cap = std::min<uint64_t>(cap, static_cast<uint64_t>(G.cfg.max_ctas));
+    const unsigned g = static_cast<unsigned>(std::max<uint64_t>(1, std::min<uint64_t>(tiles, cap)));
+#if RATEL_TMA_DYNAMIC
+    const int slot = ctr_slot(st);
+    Q.u.tile_ctr = G.d_ctr + slot;
+    Q.u.tile_base = G.ctr_base[slot];
+    G.ctr_base[slot] += tiles + g;
+#endif
+    adam_update_rs_tma_kernel<MODE, CLIP><<<g, kRsTmaThreads, rs_tma_smem_bytes(nmax), st>>>(Q);
+    return;
+  }
+#endif
   uint64_t tiles = 0;
   for (int r = 0; r < Q.u.nr; ++r) tiles += ((Q.u.r[r].n & ~7ull) + kRsTile - 1) / kRsTile;
   const unsigned g = static_cast<unsigned>(

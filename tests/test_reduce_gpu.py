@@ -56,7 +56,7 @@ def _oracle_refs(steps, world, scale, clip=0.0, sizes=SIZES):
     return refs
 
 
-def _simulate(dev, tmp_path, world, steps, pinned=False, fused=False, scale=None):
+def _simulate(dev, tmp_path, world, steps, pinned=False, fused=False, scale=None, k1_kernel=None):
     """N ranks on one GPU; returns (ranks' GpuBlocks)."""
     scale = 1.0 / world if scale is None else scale
     libs = _libs(tmp_path, world)
@@ -67,6 +67,8 @@ def _simulate(dev, tmp_path, world, steps, pinned=False, fused=False, scale=None
         L.ratel_default_config(ctypes.byref(cfg))
         cfg.comm = R.RATEL_COMM_NONE
         cfg.tile_elems = 1 << 17       # pinned: several ring tiles per slice
+        if k1_kernel is not None:
+            cfg.k1_kernel = k1_kernel
         assert L.ratel_init(0, r, world, None, ctypes.byref(cfg)) == 0, L.ratel_last_error()
         for b in ranks[r]:
             rr = (R.ratel_range * 1)(*b.ranges())
@@ -133,6 +135,19 @@ def test_fused_reduction_simulated_ranks_vs_oracle(cuda_dev, tmp_path, world, pi
         cap = R.ratel_padded_numel(n, world)
         for r in range(world):
             assert torch.count_nonzero(ranks[r][i].p16[0][n:cap].view(torch.int16)) == 0
+
+
+@pytest.mark.parametrize("world,pinned,fused", [(4, False, False), (8, False, True), (3, True, True)])
+def test_fused_reduction_tma_kernel_equals_ldg_kernel_bitwise(cuda_dev, tmp_path, world, pinned, fused):
+    """The TMA-staged K1-RS (default) and the register-staged one reduce in
+    the same fp64 rank order and run the same adam_update(): same bits."""
+    a = _simulate(cuda_dev, tmp_path, world, 2, pinned=pinned, fused=fused, k1_kernel=R.RATEL_UPDATE_TMA)
+    b = _simulate(cuda_dev, tmp_path, world, 2, pinned=pinned, fused=fused, k1_kernel=R.RATEL_UPDATE_LDG)
+    for i, n in enumerate(SIZES):
+        ga, gb = _gathered(a, i, n, world), _gathered(b, i, n, world)
+        for k in ("p32", "m32", "v32"):
+            assert np.array_equal(ga[k].view(np.uint32), gb[k].view(np.uint32)), (i, k)
+        assert np.array_equal(ga["p16"], gb["p16"])
 
 
 def test_fused_reduction_residency_bitwise(cuda_dev, tmp_path):
