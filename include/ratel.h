@@ -103,6 +103,12 @@ enum {
  *                 tile k-1 overlap.  A block's reads start when its gradient
  *                 is complete (the active message; the reader thread waits on
  *                 the hand-off event).  Single rank (no NCCL communicator). */
+/*   Hybrid (both host resources at once): register the head of a range as a
+ *                 PINNED_HOST block and the rest (a 16-byte-aligned split, the
+ *                 five pointers offset by the split) as a HOST_COMPUTE block,
+ *                 and hand both off together -- the host link and the host's
+ *                 cores then update one block concurrently (DESIGN.md §7,
+ *                 5.6-5.8 G params/s vs 4.0 / 5.1 for either alone). */
 typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2, RATEL_SSD = 3 } ratel_residency;
 typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
 /* Pinned-host staging schedule: PIPELINED = Fig. 3b (stage-in of tile k+1,
