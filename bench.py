@@ -444,7 +444,10 @@ def overlap_host_probe(args, R, torch, dev, dev_index):
     states of `--overlap-host-blocks` 13B blocks, each of a block's four linears
     registered as its own unit and handed off right after its dW GEMM (the
     paper's per-tensor hand-off), with a synthetic backward of
-    `--overlap-host-tokens` tokens.  Exposed = AGO step - backward alone."""
+    `--overlap-host-tokens` tokens.  Exposed = AGO step - backward alone.
+    Measured for the GPU-streamed residency (the north star's path) and, on the
+    same states and backward, for the paper's own CPU handler (HOST_COMPUTE).
+    Returns {residency: result}."""
     L, h = SHAPES[args.shape]
     sizes = model_blocks(args.shape, with_embedding=False)[:args.overlap_host_blocks]
     cfg = R.ratel_default_config()
@@ -461,61 +464,74 @@ def overlap_host_probe(args, R, torch, dev, dev_index):
         units.append([R.ratel_range(r0.param_bf16 + 2 * o, r0.grad_bf16 + 2 * o, 0, r0.master + 4 * o,
                                     r0.exp_avg + 4 * o, r0.exp_avg_sq + 4 * o, ln, 1) for o, ln in offs])
     K = 4
-    R.ratel_init(dev_index, 0, 1, None, cfg)
+    bw = SynthBackward(dev, h, args.overlap_host_tokens, model.p16, model.grad_ring, 0)
+    s = torch.cuda.Stream(device=dev, priority=-2)
+    order = list(reversed(range(len(sizes))))
+    P = sum(sizes)
+    out = {}
+    t_bwd = None
     try:
-        for b in range(len(sizes)):
-            for j, r in enumerate(units[b]):
-                R.ratel_register_block(b * K + j, [r], R.RATEL_PINNED_HOST)
-        bw = SynthBackward(dev, h, args.overlap_host_tokens, model.p16, model.grad_ring, 0)
-        s = torch.cuda.Stream(device=dev, priority=-2)
-        order = list(reversed(range(len(sizes))))
-        t = [1]
+        for resname, code in (("pinned-host", R.RATEL_PINNED_HOST), ("hostcompute", R.RATEL_HOST_COMPUTE)):
+            R.ratel_init(dev_index, 0, 1, None, cfg)
+            try:
+                for b in range(len(sizes)):
+                    for j, r in enumerate(units[b]):
+                        R.ratel_register_block(b * K + j, [r], code)
+                t = [1]
 
-        def bwd():
-            with torch.cuda.stream(s):
-                for b in order:
-                    bw.block(b, b % 3)
+                def bwd():
+                    with torch.cuda.stream(s):
+                        for b in order:
+                            bw.block(b, b % 3)
 
-        def opt():
-            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
-            t[0] += 1
-            for b in order:
-                for j in range(K):
-                    R.ratel_offload_grad_chunk(b * K + j, s)
-            R.ratel_sync(s)
-
-        def ago():
-            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
-            t[0] += 1
-            with torch.cuda.stream(s):
-                for jb, b in enumerate(order):
-                    if jb >= 3:
+                def opt():
+                    R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+                    t[0] += 1
+                    for b in order:
                         for j in range(K):
-                            R.ratel_block_wait((b + 3) * K + j, s)   # ring slot consumed
-                    bw.block(b, b % 3, on_linear=lambda j, b=b: R.ratel_offload_grad_chunk(b * K + j, s))
-            R.ratel_sync(s)
+                            R.ratel_offload_grad_chunk(b * K + j, s)
+                    R.ratel_sync(s)
 
-        res = {}
-        for name, fn in (("bwd", bwd), ("opt", opt), ("ago", ago)):
-            fn()
-            torch.cuda.synchronize()
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record(s)
-            for _ in range(2):
-                fn()
-            e1.record(s)
-            e1.synchronize()
-            res[name] = e0.elapsed_time(e1) / 2
-        P = sum(sizes)
-        return {"tokens": args.overlap_host_tokens, "blocks": len(sizes), "params": P,
-                "residency": "pinned-host", "handoff": "per tensor (4 linears per block)",
-                "backward_ms": res["bwd"], "optimizer_alone_ms": res["opt"], "ago_step_ms": res["ago"],
-                "exposed_optimizer_ms": res["ago"] - res["bwd"],
-                "hidden_fraction": 1.0 - (res["ago"] - res["bwd"]) / res["opt"],
-                "host_link_gbs_optimizer_alone": 24 * P / (res["opt"] / 1e3) / 1e9,
-                "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)"}
+                def ago():
+                    R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+                    t[0] += 1
+                    with torch.cuda.stream(s):
+                        for jb, b in enumerate(order):
+                            if jb >= 3:
+                                for j in range(K):
+                                    R.ratel_block_wait((b + 3) * K + j, s)   # ring slot consumed
+                            bw.block(b, b % 3, on_linear=lambda j, b=b: R.ratel_offload_grad_chunk(b * K + j, s))
+                    R.ratel_sync(s)
+
+                res = {}
+                for name, fn in (("bwd", bwd), ("opt", opt), ("ago", ago)):
+                    if name == "bwd" and t_bwd is not None:
+                        continue
+                    fn()
+                    torch.cuda.synchronize()
+                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    e0.record(s)
+                    for _ in range(2):
+                        fn()
+                    e1.record(s)
+                    e1.synchronize()
+                    res[name] = e0.elapsed_time(e1) / 2
+                t_bwd = res.get("bwd", t_bwd)
+                r = {"tokens": args.overlap_host_tokens, "blocks": len(sizes), "params": P,
+                     "residency": resname, "handoff": "per tensor (4 linears per block)",
+                     "backward_ms": t_bwd, "optimizer_alone_ms": res["opt"], "ago_step_ms": res["ago"],
+                     "exposed_optimizer_ms": res["ago"] - t_bwd,
+                     "hidden_fraction": 1.0 - (res["ago"] - t_bwd) / res["opt"],
+                     "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)"}
+                if code == R.RATEL_PINNED_HOST:
+                    r["host_link_gbs_optimizer_alone"] = 24 * P / (res["opt"] / 1e3) / 1e9
+                else:
+                    r["handler"] = "the paper's CPU AdamW (HOST_COMPUTE): G16 D2H, CPU update, P16 H2D"
+                out[resname] = r
+            finally:
+                R.ratel_finalize()
+        return out
     finally:
-        R.ratel_finalize()
         del model
         torch.cuda.empty_cache()
 
@@ -994,10 +1010,11 @@ def main():
             except Exception as ex:  # report, do not hide
                 roof = dict(roof, offdevice_error=repr(ex)[:300])
 
-        overlap_host = None
+        overlap_host = overlap_hostcompute = None
         if args.overlap_host_tokens > 0 and world == 1 and args.residency == "device":
             try:
-                overlap_host = overlap_host_probe(args, R, torch, dev, local)
+                oh = overlap_host_probe(args, R, torch, dev, local)
+                overlap_host, overlap_hostcompute = oh.get("pinned-host"), oh.get("hostcompute")
             except Exception as ex:  # report, do not hide
                 overlap_host = {"error": repr(ex)[:300]}
             torch.cuda.empty_cache()
@@ -1024,7 +1041,7 @@ def main():
                     # first timed step: issued into a drained launch queue, so this is the
                     # host cost of a step (later ones wait on queue back-pressure)
                     "host_enqueue_ms_first_step": HOST_ENQUEUE_MS[0] if HOST_ENQUEUE_MS else None,
-                    "overlap": overlap, "overlap_host": overlap_host,
+                    "overlap": overlap, "overlap_host": overlap_host, "overlap_hostcompute": overlap_hostcompute,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
             print(json.dumps(line), flush=True)
     finally:

@@ -155,6 +155,7 @@ def run(args):
 
     def init(mc, staging):
         cfg.max_ctas = mc
+        cfg.host_threads = args.host_threads
         cfg.cta_tiles = args.cta_tiles
         cfg.k1_kernel = args.k1_kernel
         if args.tile_elems:
@@ -208,7 +209,8 @@ def run(args):
                               clk.get("power_w"))
                 R.ratel_finalize()
             tb = times["bwd"][0]
-            row = {"residency": args.residency + (f" {args.hybrid_gpu_frac}" if hybrid else ""), "granularity": args.granularity, "cta_tiles": args.cta_tiles,
+            row = {"residency": args.residency + (f" {args.hybrid_gpu_frac}" if hybrid else ""),
+                   "host_threads": args.host_threads, "granularity": args.granularity, "cta_tiles": args.cta_tiles,
                    "k1_kernel": args.k1_kernel, "bwd_priority": args.bwd_priority, "ring": args.ring,
                    "tile_elems": args.tile_elems, "zero_copy": bool(args.zero_copy),
                    "tokens": tokens, "max_ctas": mc,
@@ -236,6 +238,7 @@ if __name__ == "__main__":
     ap.add_argument("--shape", default="13B")
     ap.add_argument("--blocks", type=int, default=0)
     ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute", "hybrid"])
+    ap.add_argument("--host-threads", type=int, default=0, help="cfg.host_threads (CPU handler threads, 0 = default)")
     ap.add_argument("--hybrid-gpu-frac", type=float, default=0.3,
                     help="hybrid: fraction of each unit GPU-streamed; the rest goes to the CPU handler")
     ap.add_argument("--tokens", type=int, nargs="+", default=[2048, 8192, 32768])
