@@ -130,8 +130,10 @@ typedef enum { RATEL_STAGING_PIPELINED = 0, RATEL_STAGING_SERIALIZED = 1, RATEL_
 typedef enum { RATEL_COMM_AUTO = 0, RATEL_COMM_NONE = 1, RATEL_COMM_NCCL = 2 } ratel_comm;
 
 /* Update-kernel variants (same per-element arithmetic, bitwise-identical results):
- * TMA      bulk-copy (TMA) shared-memory pipeline, one 224 KB CTA per SM, the fastest alone;
- * LDG      register-staged 128/256-bit loads, 2 CTAs per SM, no shared memory;
+ * TMA      bulk-copy (TMA) shared-memory pipeline, one 224 KB CTA per SM, the fastest alone (ranges with
+ *          peer grads, ratel_register_peer_grads: the TMA-staged fused-reduction kernel);
+ * LDG      register-staged 128/256-bit loads, 2 CTAs per SM, no shared memory (also selects the
+ *          register-staged fused-reduction kernel);
  * LDG_LITE register-staged, one octet in flight per thread, <= 64 registers, 4 CTAs per SM, no shared
  *          memory: small enough to share an SM with a backward GEMM CTA while AGO overlaps them. */
 typedef enum { RATEL_UPDATE_TMA = 0, RATEL_UPDATE_LDG = 1, RATEL_UPDATE_LDG_LITE = 2 } ratel_k1_kernel;
