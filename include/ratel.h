@@ -26,7 +26,9 @@
  *   m = b1*m + (1-b1)*g ; v = b2*v + (1-b2)*g^2
  *   theta -= lr/(1-b1^t) * m / (sqrt(v)/sqrt(1-b2^t) + eps)
  *   P16 = bf16_rne(theta)  (from the stored fp32 master)
- * fp32 math (explicit FMA placement, IEEE sqrt/div, no fast-math).
+ * fp32 math (explicit FMA placement; sqrt and 1/denominator by the <= 1-ulp
+ * sqrt.approx.f32 / rcp.approx.f32, reading R7 -- the IEEE forms are
+ * the build flag RATEL_K1_FASTMATH=0; never --use_fast_math).
  *
  * Call protocol (one host thread per process, one process per GPU; not
  * re-entrant):

@@ -12,7 +12,8 @@
 // cores.  K1 streams five SoA arrays with 128-bit loads/stores through a
 // grid-stride loop sized to the SMs, and every element -- vector body or
 // scalar tail -- goes through the SAME adam_update() with explicit
-// __fmaf_rn/__fmul_rn/__fsqrt_rn/__fdiv_rn, so the compiler cannot contract
+// __fmaf_rn/__fmul_rn (and sqrt.approx/rcp.approx, or __fsqrt_rn/__fdiv_rn with
+// RATEL_K1_FASTMATH=0; R7), so the compiler cannot contract
 // differently in the two paths.  That makes results bitwise identical across
 // world size, tile size, residency and hand-off order (R16).
 #pragma once
