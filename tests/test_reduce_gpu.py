@@ -307,3 +307,53 @@ def test_register_peer_grads_errors(cuda_dev):
         with pytest.raises(R.RatelError) as e:                              # needs a full-range grad
             R.ratel_register_peer_grads(2, 0, [None], 1.0)
         assert e.value.code == R.RATEL_EINVAL
+
+
+@pytest.mark.parametrize("k1_kernel", [R.RATEL_UPDATE_TMA, R.RATEL_UPDATE_LDG])
+def test_fused_reduction_slice_beyond_2pow32_sampled_vs_oracle(cuda_dev, k1_kernel):
+    """Maximum sizes for the fused reduction: rank 0 of a simulated world 2
+    owns a slice of 2^32 + 4104 elements of one range (both ranks' full-range
+    G16 resident here, ~103 GB in all), so the TMA-staged kernel's tile offsets
+    and the peer-grad pointers cross 2^31 and 2^32 and the slice ends in a
+    scalar tail.  Two steps; sampled elements around both boundaries and the
+    end of the slice vs the oracle's data-parallel step (R17)."""
+    n = 2 * ((1 << 32) + 4099)
+    world, scale = 2, 0.5
+    beg, end = R.ratel_rank_slice(n, world, 0)
+    s = end - beg
+    assert beg == 0 and s > (1 << 32)
+    picks = [np.arange(0, 32), np.arange((1 << 31) - 40, (1 << 31) + 40), np.arange((1 << 32) - 40, (1 << 32) + 40),
+             np.arange(s - 40, s), np.random.default_rng(6).integers(0, s, 50_000)]
+    idx = np.unique(np.concatenate(picks)).astype(np.uint64)
+    cfg = R.ratel_default_config()
+    cfg.comm = R.RATEL_COMM_NONE
+    cfg.k1_kernel = k1_kernel
+    R.ratel_init(0, 0, world, None, cfg)
+    try:
+        cap = R.ratel_padded_numel(n, world)
+        gq = [torch.empty(cap, dtype=torch.bfloat16, device=cuda_dev) for _ in range(world)]
+        th = torch.empty(s, dtype=torch.float32, device=cuda_dev)
+        R.ratel_gen_theta0(th.data_ptr(), s, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, 0))
+        m, v = torch.zeros(s, device=cuda_dev), torch.zeros(s, device=cuda_dev)
+        p = torch.zeros(cap, dtype=torch.bfloat16, device=cuda_dev)
+        R.ratel_register_block(0, [R.make_range(p, gq[0], th, m, v, n)], R.RATEL_DEVICE)
+        R.ratel_register_peer_grads(0, 0, gq, scale)
+        ref = oracle.Range.fresh(synth.theta0_at(idx, block=0))
+        for t in (1, 2):
+            for q in range(world):
+                R.ratel_gen_grad16(gq[q].data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, 1000 * q))
+            torch.cuda.synchronize()
+            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t)
+            R.ratel_offload_grad_chunk(0, None)
+            R.ratel_sync(None)
+            gd = oracle.reduce_grads([synth.grad16_at(idx, step=t, block=1000 * q) for q in range(world)], scale)
+            oracle.adam_range_gd(ref, gd, oracle.hparams(step=t, **HP))
+        ii = torch.from_numpy(idx.astype(np.int64)).to(cuda_dev)
+        got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
+                   p16=torch_to_u16(p[ii]))
+        check_range(got, ref, own_rne=oracle.bf16_rne, what=f"RS slice 2^32+ (k1_kernel {k1_kernel})")
+        assert np.array_equal(got["p16"], oracle.bf16_rne(got["p32"]))
+    finally:
+        R.ratel_finalize()
+        del gq, th, m, v, p
+        torch.cuda.empty_cache()
