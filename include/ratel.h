@@ -111,7 +111,16 @@ enum {
  *                 and hand both off together -- the host link and the host's
  *                 cores then update one block concurrently (DESIGN.md §7,
  *                 5.6-5.8 G params/s vs 4.0 / 5.1 for either alone). */
-typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2, RATEL_SSD = 3 } ratel_residency;
+/*   SSD_HOST_COMPUTE  the paper's full pipeline (Fig. 3b with its CPU
+ *                 optimizer): states in a state file exactly as RATEL_SSD
+ *                 (ratel_register_ssd), but no state crosses the host link --
+ *                 the reader thread copies the block's G16 device->host
+ *                 (2 B/param), reads each tile file -> pinned staging, runs the
+ *                 CPU AdamW on it (the HOST_COMPUTE handler) and queues it for
+ *                 the writer thread; the P16 goes host->device (2 B/param).
+ *                 Bitwise equal to HOST_COMPUTE.  Single rank. */
+typedef enum { RATEL_DEVICE = 0, RATEL_PINNED_HOST = 1, RATEL_HOST_COMPUTE = 2, RATEL_SSD = 3,
+               RATEL_SSD_HOST_COMPUTE = 4 } ratel_residency;
 typedef enum { RATEL_ADAMW = 0, RATEL_ADAM_L2 = 1 } ratel_mode;
 /* Pinned-host staging schedule: PIPELINED = Fig. 3b (stage-in of tile k+1,
  * update of tile k and write-back of tile k-1 overlap on three streams; the

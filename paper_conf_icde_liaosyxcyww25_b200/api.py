@@ -92,7 +92,7 @@ class _Range:
         flat32 = torch.cat([p.detach().reshape(-1).to(torch.float32) for p in params]).to(dev)
         s = max(end - beg, 8)
         self.ssd, self.ssd_off = ssd, None
-        if residency == "ssd":
+        if residency in ("ssd", "ssd_hostcompute"):
             # theta0 and zero moments go to the file; no state tensors are kept
             import os
             self.ssd_off = ssd.add(self.numel, world, rank)
@@ -167,7 +167,9 @@ class Ratel_Optimizer:
     the first `hybrid_gpu_frac` of every range GPU-streamed, the rest updated
     by the CPU handler -- two library blocks per unit, handed off together, so
     the host link and the host's cores work on one block at the same time;
-    single rank) or "ssd" (a state file at `ssd_path`, streamed by the
+    single rank), "ssd_hostcompute" (the paper's full pipeline: the same state
+    file, each staged tile updated by the CPU handler, no state crossing the
+    host link) or "ssd" (a state file at `ssd_path`, streamed by the
     library's reader/writer threads; the paper's storage tier, single rank).
 
     granularity: "block" hands a transformer block off when its last gradient
@@ -209,9 +211,10 @@ class Ratel_Optimizer:
                     units.append([(nodecay, False)])
         if residency == "hybrid" and world > 1:
             raise ValueError('residency="hybrid" is single-rank')
-        if residency == "ssd" and not ssd_path:
-            raise ValueError('residency="ssd" needs ssd_path (the state file to create)')
-        self.ssd = _SsdFile(ssd_path) if residency == "ssd" else None
+        ssd = residency in ("ssd", "ssd_hostcompute")
+        if ssd and not ssd_path:
+            raise ValueError(f'residency="{residency}" needs ssd_path (the state file to create)')
+        self.ssd = _SsdFile(ssd_path) if ssd else None
         for j, groups in enumerate(units):
             ranges = [_Range(ps, wd, world, rank, dev, "host" if residency == "hybrid" else residency, self.ssd)
                       for ps, wd in groups]
@@ -236,7 +239,8 @@ class Ratel_Optimizer:
             self._lib_ids[bid] = [bid]
             R.ratel_register_block(bid, [r.ratel_range() for r in ranges],
                                    {"device": R.RATEL_DEVICE, "host": R.RATEL_PINNED_HOST,
-                                    "hostcompute": R.RATEL_HOST_COMPUTE, "ssd": R.RATEL_SSD}[residency])
+                                    "hostcompute": R.RATEL_HOST_COMPUTE, "ssd": R.RATEL_SSD,
+                                    "ssd_hostcompute": R.RATEL_SSD_HOST_COMPUTE}[residency])
             if self.ssd is not None:
                 for i, r in enumerate(ranges):
                     R.ratel_register_ssd(bid, i, self.ssd.fd, r.ssd_off)

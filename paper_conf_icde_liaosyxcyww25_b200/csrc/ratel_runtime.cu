@@ -100,6 +100,7 @@ struct Block {
   };
   std::vector<SsdRange> ssd;
   uint64_t ssd_seq = 0;  // engine job number of this block's last submission
+  bool ssd_cpu = false;  // RATEL_SSD_HOST_COMPUTE: the CPU handler updates the tiles (residency stays RATEL_SSD)
 };
 
 // The SSD tier's reader/writer threads (RATEL_SSD).  Shared with the main
@@ -112,6 +113,7 @@ struct SsdJob {
 struct SsdTile {
   int slot = 0, fd = -1;
   uint64_t foff = 0, stride = 0, bytes = 0;
+  bool host = false;  // updated by the CPU handler in the staging slot (no D2H to wait for)
 };
 struct SsdEngine {
   std::thread reader, writer;
@@ -705,9 +707,100 @@ int io_full(bool rd, int fd, void* buf, uint64_t bytes, uint64_t off, std::strin
   } while (0)
 
 // One block: every tile of every range of this rank's slices.
+// RATEL_SSD_HOST_COMPUTE: the paper's own pipeline -- G16 to host, per tile
+// file -> pinned staging, the CPU handler updates it there, the writer puts it
+// back; P16 to the device at the end.  Runs on the reader thread (the CPU
+// update of a tile is an order of magnitude shorter than reading it).
+int ssd_run_job_cpu(SsdEngine& E, Block& B, std::string& msg) {
+  const uint64_t T = G.cfg.tile_elems;
+  const int D = G.cfg.pipeline_depth;
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const Slice& s = B.slices[i];
+    const uint64_t n = s.end - s.begin;
+    if (n) SK(cudaMemcpyAsync(B.h_g[i], grad_ptr(B.ranges[i], s), n * 2, cudaMemcpyDeviceToHost, E.s_in));
+  }
+  double coef = 1.0;
+  if (G.cfg.max_grad_norm > 0.0) {  // torch clip_grad_norm_: min(1, max/(||g||+1e-6)), NaN propagates
+    double S = 0.0;
+    SK(cudaStreamWaitEvent(E.s_in, G.ev_norm, 0));
+    SK(cudaMemcpyAsync(&S, G.comm != nullptr ? G.d_sumsq + 1 : G.d_sumsq, sizeof S, cudaMemcpyDeviceToHost, E.s_in));
+    SK(cudaStreamSynchronize(E.s_in));
+    const double c = G.cfg.max_grad_norm / (std::sqrt(S) + 1e-6);
+    coef = (c < 1.0 || std::isnan(c)) ? c : 1.0;
+  }
+  SK(cudaStreamSynchronize(E.s_in));  // G16 in host staging
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const ratel_range& r = B.ranges[i];
+    const Slice& s = B.slices[i];
+    const Block::SsdRange& f = B.ssd[i];
+    const uint64_t n = s.end - s.begin;
+    for (uint64_t off = 0; off < n; off += T) {
+      const uint64_t len = std::min<uint64_t>(T, n - off);
+      const int slot = static_cast<int>(E.ring_k % static_cast<uint64_t>(D));
+      {
+        std::unique_lock<std::mutex> lk(E.mu);
+        E.cv.wait(lk, [&] { return !E.slot_busy[slot] || E.err != 0; });
+        if (E.err) return E.err;
+      }
+      float* h = E.h_ring + 3ull * slot * T;
+      const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
+      const double t0 = now_s();
+      for (int a = 0; a < 3; ++a) {
+        const int rc = io_full(true, f.fd, h + a * T, bytes, f.off + a * f.stride + off * 4, msg);
+        if (rc != RATEL_OK) return rc;
+      }
+      E.read_s += now_s() - t0;
+      E.read_bytes += 3 * bytes;
+      HostAdamArgs a{};
+      a.g = B.h_g[i] + off;
+      a.th = h;
+      a.m = h + T;
+      a.v = h + 2 * T;
+      a.p = B.h_p[i] + off;
+      a.n = len;
+      a.wd_on = r.apply_weight_decay != 0;
+      a.mode = G.cfg.mode;
+      a.lr = G.hp_lr;
+      a.beta1 = G.hp_b1;
+      a.beta2 = G.hp_b2;
+      a.eps = G.hp_eps;
+      a.wd = G.hp_wd;
+      a.bc1 = G.hp_bc1;
+      a.bc2 = G.hp_bc2;
+      a.coef = coef;
+      host_adam_range(a, G.cfg.host_threads);
+      {
+        std::lock_guard<std::mutex> lk(E.mu);
+        E.slot_busy[slot] = 1;
+        SsdTile t;
+        t.slot = slot;
+        t.fd = f.fd;
+        t.foff = f.off + off * 4;
+        t.stride = f.stride;
+        t.bytes = bytes;
+        t.host = true;
+        E.wq.push_back(t);
+        ++E.tiles_in;
+      }
+      E.cv.notify_all();
+      ++E.ring_k;
+    }
+  }
+  for (size_t i = 0; i < B.ranges.size(); ++i) {
+    const Slice& s = B.slices[i];
+    const uint64_t n = s.end - s.begin;
+    if (n)
+      SK(cudaMemcpyAsync(static_cast<uint16_t*>(B.ranges[i].param_bf16) + s.begin, B.h_p[i], n * 2,
+                         cudaMemcpyHostToDevice, E.s_in));
+  }
+  SK(cudaEventRecord(B.ev_done, E.s_in));
+  return RATEL_OK;
+}
+
 int ssd_run_job(SsdEngine& E, const SsdJob& job, std::string& msg) {
   for (cudaEvent_t ev : job.wait) SK(cudaEventSynchronize(ev));  // the active message: the gradient exists
   Block& B = G.blocks[job.block];
+  if (B.ssd_cpu) return ssd_run_job_cpu(E, B, msg);
   const uint64_t T = G.cfg.tile_elems;
   const int D = G.cfg.pipeline_depth;
   bool first = true;
@@ -835,7 +928,7 @@ void ssd_writer_main(SsdEngine* E) {
     if (!failed) {
       std::string m;
       int rc = RATEL_OK;
-      const cudaError_t e = cudaEventSynchronize(E->ev_d2h[t.slot]);  // the tile's states are back in the slot
+      const cudaError_t e = t.host ? cudaSuccess : cudaEventSynchronize(E->ev_d2h[t.slot]);  // states back in the slot
       if (e != cudaSuccess) {
         rc = RATEL_ECUDA;
         m = std::string("cudaEventSynchronize(d2h) failed: ") + cudaGetErrorString(e);
@@ -1292,8 +1385,10 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
   if (ranges == nullptr || n_ranges < 1 || n_ranges > RATEL_MAX_RANGES_PER_BLOCK)
     return set_error(RATEL_EINVAL, "ratel_register_block: need 1..%d ranges", RATEL_MAX_RANGES_PER_BLOCK);
   if (residency != RATEL_DEVICE && residency != RATEL_PINNED_HOST && residency != RATEL_HOST_COMPUTE &&
-      residency != RATEL_SSD)
+      residency != RATEL_SSD && residency != RATEL_SSD_HOST_COMPUTE)
     return set_error(RATEL_EINVAL, "ratel_register_block: bad residency %d", residency);
+  const bool ssd_cpu = residency == RATEL_SSD_HOST_COMPUTE;
+  if (ssd_cpu) residency = RATEL_SSD;  // the SSD tier with the CPU handler in place of the tile kernel
   if (residency == RATEL_SSD) {
     if (G.comm != nullptr)
       return set_error(RATEL_EINVAL, "ratel_register_block: RATEL_SSD blocks need a single rank without NCCL");
@@ -1342,6 +1437,16 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
     }
   }
   Block& B = G.blocks[block_id];
+  if (ssd_cpu) {  // pinned G16 / P16 staging of the rank slices (2 + 2 B/param)
+    B.h_g.assign(n_ranges, nullptr);
+    B.h_p.assign(n_ranges, nullptr);
+    for (int i = 0; i < n_ranges; ++i) {
+      const uint64_t n = std::max<uint64_t>(8, slices[i].end - slices[i].begin);
+      CK(cudaHostAlloc(&B.h_g[i], n * 2, cudaHostAllocDefault));
+      CK(cudaHostAlloc(&B.h_p[i], n * 2, cudaHostAllocDefault));
+    }
+  }
+  B.ssd_cpu = ssd_cpu;
   if (residency == RATEL_HOST_COMPUTE) {
     if (G.h_sumsq == nullptr) {
       CK(cudaHostAlloc(&G.h_sumsq, sizeof(double), cudaHostAllocDefault));

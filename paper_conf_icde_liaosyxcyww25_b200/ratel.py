@@ -29,6 +29,7 @@ RATEL_DEVICE = 0
 RATEL_PINNED_HOST = 1
 RATEL_HOST_COMPUTE = 2
 RATEL_SSD = 3
+RATEL_SSD_HOST_COMPUTE = 4
 RATEL_ADAMW = 0
 RATEL_ADAM_L2 = 1
 RATEL_STAGING_PIPELINED = 0

@@ -102,8 +102,10 @@ class SsdBlock(GpuBlock):
     file (layout of ratel_ssd_range_bytes; the test writes theta0 and zeros
     through a buffered fd, the library gets an O_DIRECT fd)."""
 
-    def __init__(self, block_id: int, sizes, device, path, wd_flags=None, direct: bool = True, base: int = 0):
+    def __init__(self, block_id: int, sizes, device, path, wd_flags=None, direct: bool = True, base: int = 0,
+                 cpu: bool = False):
         super().__init__(block_id, sizes, device, wd_flags=wd_flags)
+        self.cpu = cpu   # RATEL_SSD_HOST_COMPUTE: the CPU handler updates the tiles
         import os
         self.path = str(path)
         self.offs_file = []
@@ -132,7 +134,7 @@ class SsdBlock(GpuBlock):
                 for i, n in enumerate(self.sizes)]
 
     def register(self):
-        R.ratel_register_block(self.id, self.ranges(), R.RATEL_SSD)
+        R.ratel_register_block(self.id, self.ranges(), R.RATEL_SSD_HOST_COMPUTE if self.cpu else R.RATEL_SSD)
         for i in range(len(self.sizes)):
             R.ratel_register_ssd(self.id, i, self.fd, self.offs_file[i])
 

@@ -201,3 +201,33 @@ def test_paper_api_ssd_residency_bitwise(cuda_dev, tmp_path):
         assert torch.equal(a, b)
     for a, b in zip(want[1], got[1]):
         assert torch.equal(a, b)
+
+
+def test_paper_api_ssd_hostcompute_equals_hostcompute(cuda_dev, tmp_path):
+    """residency="ssd_hostcompute" (states in one state file, the CPU handler on
+    each staged tile -- the paper's full pipeline) gives the same bits as the
+    CPU handler on pinned states, through the paper's API, for 3 steps."""
+    def build():
+        torch.manual_seed(4)
+        return torch.nn.Sequential(*[Block(64) for _ in range(2)]).to(cuda_dev)
+
+    x = torch.randn(32, 64, device=cuda_dev, dtype=torch.bfloat16)
+    out = []
+    for residency, kw in (("hostcompute", {}), ("ssd_hostcompute", {"ssd_path": str(tmp_path / "s.bin")})):
+        with Ratel_init(tile_elems=4096, host_threads=4):
+            model = build()
+            opt = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in model], residency=residency, **kw))
+            for _ in range(3):
+                opt.begin_step()
+                model(x).float().pow(2).mean().backward()
+                opt.end_step()
+            torch.cuda.synchronize()
+            sd = opt.state_dict()
+            out.append(([p.detach().view(torch.int16).cpu().clone() for p in model.parameters()],
+                        [t.view(torch.int32) for rs in sd["ranges"] for r in rs for t in r.values()]))
+            opt.remove_hooks()
+        opt.close()
+    for a, b in zip(out[0][0], out[1][0]):
+        assert torch.equal(a, b)
+    for a, b in zip(out[0][1], out[1][1]):
+        assert torch.equal(a, b)

@@ -54,6 +54,33 @@ def test_ssd_clip_and_multirange(cuda_dev, tmp_path):
         b.close()
 
 
+@pytest.mark.parametrize("max_norm,mode", [(0.0, oracle.ADAMW), (1e-3, oracle.ADAMW), (0.0, oracle.ADAM_L2)])
+def test_ssd_host_compute_vs_oracle_and_bitwise_host_compute(cuda_dev, tmp_path, max_norm, mode):
+    """RATEL_SSD_HOST_COMPUTE (the paper's full pipeline: states in the file,
+    G16 to host, the CPU handler on each staged tile, P16 back): within R13 of
+    the oracle at every step, and bitwise equal to HOST_COMPUTE on the same
+    inputs (same handler, same arithmetic)."""
+    sizes = [40_003, 7, 250_000]
+    ssd = [SsdBlock(0, sizes, cuda_dev, tmp_path / "a.bin", wd_flags=[1, 0, 1], cpu=True),
+           SsdBlock(1, [123_457], cuda_dev, tmp_path / "b.bin", cpu=True)]
+    run(ssd, 3, mode=mode, max_norm=max_norm, tile_elems=TILE, host_threads=4)
+    hc = [GpuBlock(0, sizes, cuda_dev, wd_flags=[1, 0, 1], host_compute=True),
+          GpuBlock(1, [123_457], cuda_dev, host_compute=True)]
+    run(hc, 3, mode=mode, max_norm=max_norm, host_threads=4)
+    assert_bitwise(snapshot(ssd), snapshot(hc))
+    for b in ssd:
+        b.close()
+
+
+def test_ssd_host_compute_mixed_residencies(cuda_dev, tmp_path):
+    """SSD + CPU handler beside GPU-updated SSD, device and pinned-host blocks in one step (random order)."""
+    blocks = [GpuBlock(0, [200_000], cuda_dev), SsdBlock(1, [300_000], cuda_dev, tmp_path / "s.bin", cpu=True),
+              SsdBlock(2, [100_003], cuda_dev, tmp_path / "t.bin"), GpuBlock(3, [100_000], cuda_dev, pinned=True)]
+    run(blocks, 3, order="random", max_norm=5e-3, tile_elems=TILE)
+    for b in blocks[1:3]:
+        b.close()
+
+
 def test_ssd_mixed_with_device_and_pinned(cuda_dev, tmp_path):
     blocks = [GpuBlock(0, [200_000], cuda_dev), SsdBlock(1, [300_000], cuda_dev, tmp_path / "s.bin"),
               GpuBlock(2, [100_000], cuda_dev, pinned=True)]

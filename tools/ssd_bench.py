@@ -101,6 +101,8 @@ def main():
     ap.add_argument("--depths", default="2,4,8")
     ap.add_argument("--tile-elems", type=int, default=0)
     ap.add_argument("--probe-gb", type=float, default=8.0)
+    ap.add_argument("--handlers", default="gpu,cpu",
+                    help="gpu: RATEL_SSD (tile kernel); cpu: RATEL_SSD_HOST_COMPUTE (the paper's CPU handler)")
     args = ap.parse_args()
 
     import torch
@@ -112,7 +114,8 @@ def main():
     dev = torch.device("cuda:0")
     sizes = model_blocks(args.shape)[:args.blocks]
     path = os.path.join(args.dir, "ratel_ssd_states.bin")
-    for depth in (int(x) for x in args.depths.split(",")):
+    runs = [(d, h) for h in args.handlers.split(",") for d in (int(x) for x in args.depths.split(","))]
+    for depth, handler in runs:
         cfg = R.ratel_default_config()
         cfg.pipeline_depth = depth
         if args.tile_elems:
@@ -145,7 +148,8 @@ def main():
             fd = os.open(path, os.O_RDWR | os.O_DIRECT)
             fds.append(fd)
             for b, n in enumerate(sizes):
-                R.ratel_register_block(b, [R.make_range(p16[b], g16[b], None, None, None, n)], R.RATEL_SSD)
+                R.ratel_register_block(b, [R.make_range(p16[b], g16[b], None, None, None, n)],
+                                       R.RATEL_SSD_HOST_COMPUTE if handler == "cpu" else R.RATEL_SSD)
                 R.ratel_register_ssd(b, 0, fd, offs[b])
             s = torch.cuda.Stream(device=dev)
             order = list(reversed(range(len(sizes))))
@@ -171,7 +175,7 @@ def main():
             P = sum(sizes)
             gbs = 24.0 * P / dt / 1e9
             print(json.dumps({
-                "residency": "ssd", "shape": args.shape, "blocks": len(sizes), "params": P,
+                "residency": "ssd" if handler == "gpu" else "ssd_host_compute", "shape": args.shape, "blocks": len(sizes), "params": P,
                 "pipeline_depth": depth, "tile_elems": int(cfg.tile_elems), "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": dt * 1e3, "params_per_s": P / dt,
                 "ssd_gbs_24B_per_param": gbs, "roofline_gbs": probe.get("roofline_gbs"),
