@@ -595,6 +595,7 @@ void CUDART_CB host_adam_cb(void* arg) {
   if (t->sumsq != nullptr) {  // torch clip_grad_norm_: min(1, max/(||g||+1e-6)), NaN propagates
     const double c = t->max_norm / (std::sqrt(*t->sumsq) + 1e-6);
     coef = (c < 1.0 || std::isnan(c)) ? c : 1.0;
+    if (!std::isfinite(*t->sumsq)) *G.h_flag = 1;  // reported by a blocking ratel_sync (no kernel may see it)
   }
   for (HostAdamArgs& a : t->ranges) {
     a.coef = coef;
@@ -727,6 +728,7 @@ int ssd_run_job_cpu(SsdEngine& E, Block& B, std::string& msg) {
     SK(cudaStreamSynchronize(E.s_in));
     const double c = G.cfg.max_grad_norm / (std::sqrt(S) + 1e-6);
     coef = (c < 1.0 || std::isnan(c)) ? c : 1.0;
+    if (!std::isfinite(S)) *G.h_flag = 1;  // reported by a blocking ratel_sync
   }
   SK(cudaStreamSynchronize(E.s_in));  // G16 in host staging
   for (size_t i = 0; i < B.ranges.size(); ++i) {

@@ -339,8 +339,12 @@ def test_protocol_errors(cuda_dev):
     assert e.value.code == R.RATEL_ESTATE
 
 
-def test_nonfinite_norm_reported(cuda_dev):
-    b = GpuBlock(0, [4096], cuda_dev)
+@pytest.mark.parametrize("residency", ["device", "host_compute"])
+def test_nonfinite_norm_reported(cuda_dev, residency):
+    """A NaN gradient under clipping: the blocking sync reports RATEL_ENONFINITE
+    and the NaN coefficient propagates (torch), also when only the CPU handler
+    updates (no kernel sees the norm)."""
+    b = GpuBlock(0, [4096], cuda_dev, host_compute=(residency == "host_compute"))
     with ratel_lib(max_grad_norm=1.0):
         b.register()
         g = b.grads_np(1)[0].copy()

@@ -171,3 +171,22 @@ def test_ssd_io_error_is_sticky(cuda_dev, tmp_path):
     with ratel_lib(tile_elems=TILE):                    # finalize cleared it
         pass
     b.close()
+
+
+def test_ssd_host_compute_nonfinite_norm_reported(cuda_dev, tmp_path):
+    """SSD + CPU handler under clipping with a NaN gradient: RATEL_ENONFINITE
+    from the blocking sync, NaN propagated into the file's states."""
+    b = SsdBlock(0, [70_000], cuda_dev, tmp_path / "n.bin", cpu=True)
+    with ratel_lib(max_grad_norm=1.0, tile_elems=TILE):
+        b.register()
+        g = b.grads_np(1)[0].copy()
+        g[5] = 0x7FC0
+        b.g16[0][:70_000].copy_(torch.from_numpy(g.view(np.int16)).to(cuda_dev).view(torch.bfloat16))
+        torch.cuda.synchronize()
+        R.ratel_adam_step(1e-3, 0.9, 0.999, 1e-8, 1e-2, 1)
+        R.ratel_offload_grad_chunk(0, None)
+        with pytest.raises(R.RatelError) as e:
+            R.ratel_sync(None)
+        assert e.value.code == R.RATEL_ENONFINITE
+    assert np.isnan(b.gpu_state(0)["p32"]).all()
+    b.close()
