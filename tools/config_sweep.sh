@@ -18,4 +18,6 @@ run --shape c1 --steps 200 --warmup 10
 # the hybrid residency (30 % GPU-streamed + 70 % CPU handler) on the C4 / C5 shapes
 run --shape 70B --residency hybrid --blocks 3 --steps 3 --warmup 3
 run --shape 175B --residency hybrid --blocks 2 --steps 3 --warmup 3
+# per-rank HBM work of C3 at N = 8 / 4 (rank 0 of a simulated world, no collectives)
+timeout 900 python tools/rank_sim.py --shape 30B --worlds 8 4 --clip 1.0 > gpurun_out/rank_sim.jsonl 2>> gpurun_out/configs_err.log
 echo done
