@@ -167,7 +167,8 @@ class Ratel_Optimizer:
     the first `hybrid_gpu_frac` of every range GPU-streamed, the rest updated
     by the CPU handler -- two library blocks per unit, handed off together, so
     the host link and the host's cores work on one block at the same time;
-    single rank), "ssd_hostcompute" (the paper's full pipeline: the same state
+    single rank; unit j uses library block ids first_block_id + j and
+    first_block_id + len(units) + j), "ssd_hostcompute" (the paper's full pipeline: the same state
     file, each staged tile updated by the CPU handler, no state crossing the
     host link) or "ssd" (a state file at `ssd_path`, streamed by the
     library's reader/writer threads; the paper's storage tier, single rank).
