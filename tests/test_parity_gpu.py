@@ -919,3 +919,44 @@ def test_graph_capture_is_refused_without_side_effects(cuda_dev):
         R.ratel_sync(None)
     oracle.adam_step(b.oracle, gs, oracle.hparams(step=1, **HP))
     check_range(b.gpu_state(0), b.oracle[0], own_rne=oracle.bf16_rne, what="after refused capture")
+
+
+def test_long_run_300_steps_with_schedule_sampled_vs_oracle(cuda_dev):
+    """A long run: one 13B-shaped block, 300 AGO steps with a warm-up + cosine
+    lr schedule and weight decay, a fresh device-generated gradient every
+    step.  Rounding errors must not accumulate past R13: sampled elements vs
+    the oracle after steps 10, 100 and 300 (the oracle runs the same 300
+    steps on the samples); P16 == bf16(P32) everywhere at the end."""
+    h = 5120
+    n = 12 * h * h + 13 * h
+    idx = np.unique(np.concatenate([np.arange(0, 64), np.arange(n - 64, n),
+                                    np.random.default_rng(8).integers(0, n, 50_000)])).astype(np.uint64)
+
+    def lr_at(t, peak=3e-4, warm=30, total=300):
+        if t <= warm:
+            return peak * t / warm
+        return 0.5 * peak * (1 + math.cos(math.pi * (t - warm) / (total - warm))) + 1e-6
+
+    ii = torch.from_numpy(idx.astype(np.int64)).to(cuda_dev)
+    with ratel_lib():
+        g = torch.empty(n, dtype=torch.bfloat16, device=cuda_dev)
+        th = torch.empty(n, dtype=torch.float32, device=cuda_dev)
+        R.ratel_gen_theta0(th.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_THETA, 0, 0))
+        m, v = torch.zeros(n, device=cuda_dev), torch.zeros(n, device=cuda_dev)
+        p = torch.zeros(n, dtype=torch.bfloat16, device=cuda_dev)
+        R.ratel_register_block(0, [R.make_range(p, g, th, m, v, n)], R.RATEL_DEVICE)
+        ref = oracle.Range.fresh(synth.theta0_at(idx, block=0))
+        for t in range(1, 301):
+            lr = lr_at(t)
+            R.ratel_adam_step(lr, 0.9, 0.95, 1e-8, 0.1, t)
+            R.ratel_block_wait(0, None)   # the grad buffer is rewritten every step
+            R.ratel_gen_grad16(g.data_ptr(), n, 0, R.ratel_gen_stream_key(synth.SEED, synth.TAG_GRAD, t, 0))
+            R.ratel_offload_grad_chunk(0, None)
+            R.ratel_sync(None)
+            oracle.adam_range(ref, synth.grad16_at(idx, step=t, block=0),
+                              oracle.hparams(lr=lr, beta1=0.9, beta2=0.95, eps=1e-8, weight_decay=0.1, step=t))
+            if t in (10, 100, 300):
+                got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
+                           p16=torch_to_u16(p[ii]))
+                check_range(got, ref, own_rne=oracle.bf16_rne, what=f"long run step {t}")
+        assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
