@@ -958,5 +958,6 @@ def test_long_run_300_steps_with_schedule_sampled_vs_oracle(cuda_dev):
             if t in (10, 100, 300):
                 got = dict(p32=th[ii].cpu().numpy(), m32=m[ii].cpu().numpy(), v32=v[ii].cpu().numpy(),
                            p16=torch_to_u16(p[ii]))
-                check_range(got, ref, own_rne=oracle.bf16_rne, what=f"long run step {t}")
+                rep = check_range(got, ref, own_rne=oracle.bf16_rne, what=f"long run step {t}")
+                print(f"long run step {t}: {rep}")
         assert torch.equal(p.view(torch.int16), th.to(torch.bfloat16).view(torch.int16))
