@@ -21,7 +21,8 @@ model's parameters become bf16 views of P16 and their ``.grad`` views of G16,
 so autograd accumulates straight into the buffers the library reads.  The
 hand-off is a post-accumulate-grad hook with a per-block countdown.  All
 arithmetic is in libratel.so; this module only arranges memory and calls.
-One backward per step (no gradient accumulation across micro-batches).
+Gradient accumulation: begin_step(micro_batches=k) hands units off during the
+k-th backward.
 """
 from __future__ import annotations
 
@@ -248,6 +249,7 @@ class Ratel_Optimizer:
         self._pending = {}
         self._handed = set()
         self._hooks = []
+        self._micro = 1
 
     # ------------------------------------------------------------ Ratel_hook
     def install_hooks(self):
@@ -258,7 +260,7 @@ class Ratel_Optimizer:
 
     def _make_hook(self, bid, count):
         def hook(_p):
-            left = self._pending.get(bid, count) - 1
+            left = self._pending.get(bid, count * self._micro) - 1
             self._pending[bid] = left
             if left == 0 and bid not in self._handed:
                 self._handed.add(bid)
@@ -268,8 +270,15 @@ class Ratel_Optimizer:
         return hook
 
     # ------------------------------------------------------------- a step
-    def begin_step(self, lr=None, weight_decay=None):
-        """Zero the grad buffers and arm step t (before backward = AGO)."""
+    def begin_step(self, lr=None, weight_decay=None, micro_batches=1):
+        """Zero the grad buffers and arm step t (before backward = AGO).
+        micro_batches > 1: gradient accumulation -- the step's gradients are
+        the sum over that many backward passes, and each unit is handed off
+        when its last parameter's gradient of the LAST micro-batch has
+        accumulated (only that backward overlaps the update)."""
+        if micro_batches < 1:
+            raise ValueError("micro_batches must be >= 1")
+        self._micro = int(micro_batches)
         for ranges in self.blocks:
             for r in ranges:
                 r.g16.zero_()

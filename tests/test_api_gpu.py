@@ -231,3 +231,40 @@ def test_paper_api_ssd_hostcompute_equals_hostcompute(cuda_dev, tmp_path):
         assert torch.equal(a, b)
     for a, b in zip(out[0][1], out[1][1]):
         assert torch.equal(a, b)
+
+
+def test_paper_api_gradient_accumulation_matches_oracle(cuda_dev):
+    """begin_step(micro_batches=2): autograd accumulates two backward passes
+    into the flat G16 buffers; every unit is handed off during the second
+    one (not the first), and the update equals the oracle on the accumulated
+    gradient."""
+    torch.manual_seed(5)
+    d, nb = 64, 2
+    model = torch.nn.Sequential(*[Block(d) for _ in range(nb)]).to(cuda_dev)
+    hp = dict(lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, weight_decay=0.01)
+    xs = [torch.randn(16, d, device=cuda_dev, dtype=torch.bfloat16) for _ in range(2)]
+    with Ratel_init():
+        opt = Ratel_hook(Ratel_Optimizer([list(b.parameters()) for b in model], lr=hp["lr"],
+                                         weight_decay=hp["weight_decay"]))
+        refs = []
+        for bi in range(nb):
+            for (master, m, v, p16, g16), rng in zip(opt.state(bi), opt.blocks[bi]):
+                refs.append((rng, oracle.Range.fresh(master[:rng.numel].cpu().numpy(), int(rng.apply_wd))))
+        for t in (1, 2):
+            opt.begin_step(micro_batches=2)
+            model(xs[0]).float().pow(2).mean().backward()
+            torch.cuda.synchronize()
+            assert len(opt._handed) == 0                 # nothing handed off after the first micro-batch
+            model(xs[1]).float().pow(2).mean().backward()
+            torch.cuda.synchronize()
+            assert len(opt._handed) == nb
+            grads = [r.g16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16) for r, _ in refs]
+            opt.end_step()
+            torch.cuda.synchronize()
+            for (rng, ref), g in zip(refs, grads):
+                oracle.adam_range(ref, g, oracle.hparams(step=t, **hp))
+                got = dict(p32=rng.master[:rng.numel].cpu().numpy(), m32=rng.m[:rng.numel].cpu().numpy(),
+                           v32=rng.v[:rng.numel].cpu().numpy(),
+                           p16=rng.p16[:rng.numel].view(torch.int16).cpu().numpy().view(np.uint16))
+                check_range(got, ref, own_rne=oracle.bf16_rne, what=f"accumulation step {t}")
+        opt.remove_hooks()
