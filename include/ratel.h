@@ -110,7 +110,7 @@ enum {
  *                 five pointers offset by the split) as a HOST_COMPUTE block,
  *                 and hand both off together -- the host link and the host's
  *                 cores then update one block concurrently (DESIGN.md §7,
- *                 5.6-5.8 G params/s vs 4.0 / 5.1 for either alone). */
+ *                 5.6-6.1 G params/s vs 4.0 / 5.1-5.3 for either alone). */
 /*   SSD_HOST_COMPUTE  the paper's full pipeline (Fig. 3b with its CPU
  *                 optimizer): states in a state file exactly as RATEL_SSD
  *                 (ratel_register_ssd), but no state crosses the host link --
