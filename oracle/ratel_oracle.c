@@ -35,7 +35,10 @@
  * Build: gcc -O2 -ffp-contract=off -fopenmp -fPIC -shared (no -ffast-math, no
  * FMA contraction: the double arithmetic is exactly the C expression order).
  * Pinned by tests/test_oracle_pins.py (closed forms, invariants, torch float64
- * AdamW/Adam/clip_grad_norm_, a 50-digit mpmath trace, exhaustive bf16 RNE).
+ * AdamW/Adam/clip_grad_norm_, a 50-digit mpmath trace, exhaustive bf16 RNE);
+ * the scales by tests/test_oracle_scale_pins.py (step-1 and constant-gradient
+ * closed forms, zero-gradient decay, |theta| <= theta_bar and |m| <= m_bar,
+ * the Cauchy-Schwarz bound on each step, a 50-digit trace of both scales).
  */
 #include <math.h>
 #include <stddef.h>

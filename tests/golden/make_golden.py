@@ -25,7 +25,9 @@ C1_SIZES = [H, H, 3 * H * H, 3 * H, H * H, H, H, H, 4 * H * H, 4 * H, 4 * H * H,
 C1_WD = [0, 0, 1, 0, 1, 0, 0, 0, 1, 0, 1, 0]
 
 
-def run(case):
+def run(case, scales=False):
+    """Digest of the fp32/bf16 outputs, or (scales=True) of the tolerance
+    scales theta_bar / m_bar the oracle tracks beside them (R13)."""
     n = sum(C1_SIZES)
     th0 = synth.theta0(n, block=0)
     offs = np.concatenate([[0], np.cumsum(C1_SIZES)])
@@ -41,7 +43,7 @@ def run(case):
                          max_grad_norm=case["clip"])
     h = hashlib.sha256()
     for r in ranges:
-        for a in (r.p32, r.m32, r.v32, r.p16):
+        for a in ((r.theta_bar, r.m_bar) if scales else (r.p32, r.m32, r.v32, r.p16)):
             h.update(np.ascontiguousarray(a).tobytes())
     return h.hexdigest()
 
@@ -58,10 +60,15 @@ def digests():
     return {k: run(v) for k, v in CASES.items()}
 
 
+def scale_digests():
+    return {k: run(v, scales=True) for k, v in CASES.items()}
+
+
 if __name__ == "__main__":
     out = {"source": "tests/golden/make_golden.py (oracle/ + synth/ only)",
            "workload": "C1: one GPT block h=256 (789,760 params), 10 steps, torch-default hyperparameters",
-           "sha256": digests()}
+           "sha256": digests(),
+           "sha256_scales": scale_digests()}
     with open(os.path.join(HERE, "oracle_digests.json"), "w") as f:
         json.dump(out, f, indent=1)
     print(json.dumps(out, indent=1))

@@ -45,14 +45,36 @@ MUTANTS = {
     "dp_drops_last_rank": ("for (int q = 0; q < nq; ++q)", "for (int q = 0; q < nq - 1; ++q)"),
     "dp_ignores_clip_coef": ("double g = gd[i] * coef;", "double g = gd[i];"),
     "dp_sumsq_abs": ("s += g[i] * g[i];", "s += fabs(g[i]);"),
+    # tolerance scales theta_bar / m_bar (R13): every parity bound divides by them
+    "theta_bar_x2": ("theta_bar[i] = d * theta_bar[i] + absdelta;",
+                     "theta_bar[i] = 2.0 * (d * theta_bar[i] + absdelta);"),
+    "theta_bar_x100_delta": ("theta_bar[i] = d * theta_bar[i] + absdelta;",
+                             "theta_bar[i] = d * theta_bar[i] + 100.0 * absdelta;"),
+    "theta_bar_no_decay": ("double d = (apply_wd && hp->mode == ORACLE_ADAMW) ? (1.0 - hp->lr * hp->weight_decay) : 1.0;",
+                           "double d = 1.0;"),
+    "theta_bar_decay_in_l2_mode": ("double d = (apply_wd && hp->mode == ORACLE_ADAMW) ? (1.0 - hp->lr * hp->weight_decay) : 1.0;",
+                                   "double d = apply_wd ? (1.0 - hp->lr * hp->weight_decay) : 1.0;"),
+    "theta_bar_drops_delta": ("theta_bar[i] = d * theta_bar[i] + absdelta;", "theta_bar[i] = d * theta_bar[i];"),
+    "theta_bar_signed_delta": ("return fabs(delta);", "return delta;"),
+    "m_bar_no_beta1_decay": ("m_bar[i] = hp->beta1 * m_bar[i] + (1.0 - hp->beta1) * fabs(g_used);",
+                             "m_bar[i] = m_bar[i] + (1.0 - hp->beta1) * fabs(g_used);"),
+    "m_bar_signed_g": ("(1.0 - hp->beta1) * fabs(g_used);", "(1.0 - hp->beta1) * g_used;"),
+    "m_bar_drops_1_minus_beta1": ("(1.0 - hp->beta1) * fabs(g_used);", "fabs(g_used);"),
+    "m_bar_uses_beta2": ("m_bar[i] = hp->beta1 * m_bar[i] + (1.0 - hp->beta1) * fabs(g_used);",
+                         "m_bar[i] = hp->beta2 * m_bar[i] + (1.0 - hp->beta2) * fabs(g_used);"),
+    "m_bar_l2_from_raw_grad": [("double th = *theta;", "double th = *theta;\n  *g_used = g;"),
+                               ("  *g_used = g;\n  return fabs(delta);", "  return fabs(delta);")],
 }
 
 
-def _build_mutant(tmp_path, name, old, new):
+def _build_mutant(tmp_path, name, edits):
+    """edits: one (old, new) pair or a list of them, applied in order."""
     src = open(SRC).read()
-    assert src.count(old) >= 1, (name, old)  # every occurrence is mutated
+    for old, new in ([edits] if isinstance(edits, tuple) else edits):
+        assert src.count(old) >= 1, (name, old)  # every occurrence is mutated
+        src = src.replace(old, new)
     path = tmp_path / f"{name}.c"
-    path.write_text(src.replace(old, new))
+    path.write_text(src)
     so = tmp_path / f"lib{name}.so"
     subprocess.check_call(["gcc", "-O2", "-ffp-contract=off", "-fopenmp", "-fPIC", "-shared", "-std=c11",
                            "-o", str(so), str(path), "-lm"])
@@ -103,6 +125,31 @@ def _pins_pass():
             oracle.adam_range(r, cb, oracle.hparams(step=t, weight_decay=0.0))
         exp = np.array([0.01, -0.02, 0.03, 0.0]) - 10 * lr * vals / (np.abs(vals.astype(np.float64)) + eps)
         if not np.all(np.abs(r.p32 - exp) <= 10 * f32ulp(np.abs(exp) + 10 * lr)):
+            return False
+        # tolerance scales (tests/test_oracle_scale_pins.py): step-1 closed forms, AdamW and Adam-L2
+        for mode, wd in ((oracle.ADAMW, 1e-2), (oracle.ADAM_L2, 1e-2)):
+            r = oracle.Range.fresh(th0)
+            oracle.adam_range(r, g, oracle.hparams(step=1, weight_decay=wd, mode=mode))
+            gu = synth.bf16_bits_to_f32(g).astype(np.float64)
+            d = 1 - lr * wd
+            if mode == oracle.ADAM_L2:
+                gu, d = gu + wd * th0.astype(np.float64), 1.0
+            if not np.all(np.abs(r.m_bar - 0.1 * np.abs(gu)) <= 1e-15 * np.abs(gu)):
+                return False
+            exp = d * np.abs(th0.astype(np.float64)) + lr * np.abs(gu) / (np.abs(gu) + eps)
+            if not np.all(np.abs(r.theta_bar - exp) <= 2.0 ** -21 * exp):
+                return False
+        # scales under a constant gradient: m_bar = |c|(1-b1^t), theta_bar = |theta0| + t lr |c|/(|c|+eps)
+        vals = np.array([2.0 ** -10, -(2.0 ** -20), 3 * 2.0 ** -15, -(2.0 ** -8)], np.float32)
+        cb = (vals.view(np.uint32) >> 16).astype(np.uint16)
+        r = oracle.Range.fresh(np.array([0.01, -0.02, 0.03, 0.0], np.float32))
+        for t in range(1, 6):
+            oracle.adam_range(r, cb, oracle.hparams(step=t, weight_decay=0.0))
+        c = np.abs(vals.astype(np.float64))
+        if not np.all(np.abs(r.m_bar - c * (1 - 0.9 ** 5)) <= 1e-14 * c):
+            return False
+        exp = np.array([0.01, 0.02, 0.03, 0.0], np.float32).astype(np.float64) + 5 * lr * c / (c + eps)
+        if not np.all(np.abs(r.theta_bar - exp) <= 2.0 ** -18 * exp):
             return False
         # torch.optim.AdamW, 10 steps, fp32 storage emulated (R13 bound 1e-6)
         from tests.tolerance import check_range
@@ -172,8 +219,7 @@ def test_unmutated_oracle_passes_the_compact_pins():
 
 @pytest.mark.parametrize("name", sorted(MUTANTS))
 def test_every_mutant_is_caught(tmp_path, name):
-    old, new = MUTANTS[name]
-    so = _build_mutant(tmp_path, name, old, new)
+    so = _build_mutant(tmp_path, name, MUTANTS[name])
     saved = _with_lib(so)
     try:
         assert not _pins_pass(), f"mutant {name} survived the pins"

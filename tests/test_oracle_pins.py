@@ -296,8 +296,9 @@ def test_oracle_regression_digests():
     spec = importlib.util.spec_from_file_location("make_golden", os.path.join(here, "make_golden.py"))
     mg = importlib.util.module_from_spec(spec)
     spec.loader.exec_module(mg)
-    want = json.load(open(os.path.join(here, "oracle_digests.json")))["sha256"]
-    assert mg.digests() == want
+    gold = json.load(open(os.path.join(here, "oracle_digests.json")))
+    assert mg.digests() == gold["sha256"]
+    assert mg.scale_digests() == gold["sha256_scales"]   # theta_bar / m_bar (R13)
 
 
 # ------------------------------------- data-parallel gradient reduction (R17)
