@@ -152,19 +152,66 @@ def gpu_uuid(torch, dev):
 
 
 # ------------------------------------------------------ reference arm (oracle)
-def oracle_sample_rate(n: int, steps: int, threads: int, min_seconds: float = 0.0):
-    """Time the CPU oracle's update over an n-element sample of block 0 of the
-    workload (inputs generated outside the timed region)."""
-    import numpy as np
+def cpu_facts():
+    """Host CPU model, socket and NUMA-node counts (the oracle's machine)."""
+    model, sockets = None, set()
+    try:
+        with open("/proc/cpuinfo") as f:
+            for line in f:
+                k, _, v = line.partition(":")
+                k = k.strip()
+                if k == "model name" and model is None:
+                    model = v.strip()
+                elif k == "physical id":
+                    sockets.add(v.strip())
+    except OSError:
+        pass
+    try:
+        numa = len([d for d in os.listdir("/sys/devices/system/node") if d.startswith("node") and d[4:].isdigit()])
+    except OSError:
+        numa = None
+    return {"cpu_model": model, "sockets": len(sockets) or None, "numa_nodes": numa, "nproc": os.cpu_count()}
+
+
+_ORACLE_INPUTS = {}
+
+
+def oracle_inputs(n: int):
+    """theta0 and two bf16 gradient draws of an n-element sample of block 0
+    (synth/, the seeded recipe).  Large samples repeat a 2^25-element draw
+    (the generator is numpy: ~1 s per 2^25 draws, so drawing a whole 13B
+    block would take longer than timing it); only the update is timed."""
+    if n not in _ORACLE_INPUTS:
+        import numpy as np
+        import synth
+        k = min(n, 1 << 25)
+        th = synth.theta0(k, block=0)
+        gs = [synth.grad16(k, step=t, block=0) for t in (1, 2)]
+        if n > k:
+            reps = -(-n // k)
+            th = np.tile(th, reps)[:n]
+            gs = [np.tile(g, reps)[:n] for g in gs]
+        _ORACLE_INPUTS.clear()
+        _ORACLE_INPUTS[n] = (th, gs)
+    return _ORACLE_INPUTS[n]
+
+
+def oracle_sample_rate(n: int, steps: int, threads: int, min_seconds: float = 0.0, warmup: int = 1):
+    """Time the CPU oracle's update (oracle/, as it stands) over an n-element
+    sample of block 0 of the workload: `warmup` untimed passes (first touch),
+    then at least `steps` timed passes and `min_seconds`.  Returns
+    (params/s, passes, seconds)."""
     import oracle
-    import synth
-    r = oracle.Range.fresh(synth.theta0(n, block=0))
-    r.theta_bar = r.m_bar = None
-    grads = [synth.grad16(n, step=t, block=0) for t in range(1, 3)]
-    oracle.adam_range(r, grads[0], oracle.hparams(step=1), threads=threads)  # warm / first-touch
-    done, t0, t = 0, time.perf_counter(), 2
+    th, gs = oracle_inputs(n)
+    r = oracle.Range.fresh(th)
+    r.theta_bar = r.m_bar = None          # the product's 28 B/param, no tolerance scales
+    t = 1
+    for _ in range(warmup):
+        oracle.adam_range(r, gs[t % 2], oracle.hparams(step=t), threads=threads)
+        t += 1
+    done, t0 = 0, time.perf_counter()
     while done < steps or (time.perf_counter() - t0) < min_seconds:
-        oracle.adam_range(r, grads[t % 2], oracle.hparams(step=t), threads=threads)
+        oracle.adam_range(r, gs[t % 2], oracle.hparams(step=t), threads=threads)
         done += 1
         t += 1
     dt = time.perf_counter() - t0
@@ -178,24 +225,38 @@ def host_threads():
         return os.cpu_count() or 1
 
 
+def oracle_baseline(n: int, steps: int, warmup: int, threads: int, min_seconds: float = 0.0):
+    """cpu_baseline object: the oracle on an n-element sample at `threads`
+    threads, with the host facts and the DRAM rate its 28 B/param imply."""
+    v, done, dt = oracle_sample_rate(n, steps, threads, min_seconds=min_seconds, warmup=warmup)
+    out = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
+           "sample": f"{n:,} params of block 0 (one 13B block = 314,639,360), {done} timed passes in {dt:.2f} s "
+                     f"after {warmup} untimed, OpenMP {threads} threads",
+           "sample_params": n, "sample_passes": done, "sample_ms_per_pass": 1e3 * dt / done,
+           "dram_gbs_at_28B_per_param": 28 * v / 1e9}
+    out.update(cpu_facts())
+    return out
+
+
 def run_reference(args, rank, world):
+    """The reference arm: the oracle as it stands on this host's cores.  One
+    step = one oracle pass over a bounded sample of the workload (default
+    one whole 13B block); ms_per_step is that pass, as timed."""
     if rank != 0:
-        return
+        return                               # under torchrun rank 0 alone runs and prints
     n = args.oracle_sample
     threads = host_threads()
-    steps = args.steps
-    # warmup steps: untimed oracle passes
-    oracle_sample_rate(n, max(1, args.warmup), threads)
-    v, done, dt = oracle_sample_rate(n, steps, threads)
+    cb = oracle_baseline(n, args.steps, args.warmup, threads)
+    v = cb["value"]
     cfg = workload_config(args, world)
-    sample = (f"{n:,} params of block 0 of the {cfg['workload']} (one 13B-block slice), "
-              f"{done} steps, {threads} threads")
     print(json.dumps({
         "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
-        "steps": done, "warmup": args.warmup, "ms_per_step": 1e3 * dt / done * (cfg["params"] / n),
-        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-        "data": "synthetic", "config": cfg,
-        "cpu_baseline": {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle", "sample": sample},
+        "steps": cb["sample_passes"], "warmup": args.warmup, "ms_per_step": cb["sample_ms_per_pass"],
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
+        "dtype": "f64", "data": "synthetic", "config": cfg,
+        "step": f"one oracle pass over a {n:,}-param sample of the workload ({cfg['params']:,} params)",
+        "full_workload_ms_per_step_extrapolated": 1e3 * cfg["params"] / v,
+        "cpu_baseline": cb,
         "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }), flush=True)
 
@@ -810,9 +871,56 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
 
 
 # ------------------------------------------------------------------- main
+def free_port() -> int:
+    import socket
+    with socket.socket() as so:
+        so.bind(("127.0.0.1", 0))
+        return so.getsockname()[1]
+
+
+def relaunch_or_world(args) -> int:
+    """World size of this run.  `--gpus N` (N > 1) outside torchrun re-executes
+    this script under torch.distributed.run with N ranks on this node (master
+    127.0.0.1) and exits with its return code, so `python bench.py --gpus 8`
+    can never silently measure one GPU; under torchrun WORLD_SIZE must equal
+    --gpus (rc 2 otherwise)."""
+    env_world = os.environ.get("WORLD_SIZE")
+    if env_world is None:
+        n = args.gpus or 1
+        if n > 1:
+            cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+                   "--master-addr", "127.0.0.1", f"--master-port={free_port()}",
+                   os.path.abspath(__file__)] + sys.argv[1:]
+            print(f"bench.py: --gpus {n}: re-launching under torch.distributed.run ({n} ranks)",
+                  file=sys.stderr, flush=True)
+            sys.stdout.flush()
+            rc = subprocess.call(cmd)
+            raise SystemExit(rc)
+        return 1
+    world = int(env_world)
+    if args.gpus is not None and args.gpus != world:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}: refusing to measure a different "
+              f"number of GPUs than asked", file=sys.stderr, flush=True)
+        raise SystemExit(2)
+    return world
+
+
+def share_gpu_nccl_env(rank: int) -> None:
+    """--share-gpu: NCCL refuses two ranks on one device of one host ("Duplicate
+    GPU"); giving each rank its own NCCL host id makes them peers on different
+    "hosts" that talk over loopback sockets, so the real NCCL data path (the
+    library's all-gather / allreduce, torch's process group) runs with N ranks
+    on the one GPU a gpurun box has.  Set before any communicator exists."""
+    os.environ["NCCL_HOSTID"] = f"ratel-bench-rank{rank}"
+    os.environ.setdefault("NCCL_SOCKET_IFNAME", "lo")
+    os.environ.setdefault("NCCL_IB_DISABLE", "1")
+
+
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--gpus", type=int, default=None,
+                    help="N GPUs of this node; N > 1 without torchrun re-launches this script under "
+                         "torch.distributed.run (one rank per GPU); under torchrun it must equal WORLD_SIZE")
     ap.add_argument("--steps", type=int, default=20)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ratel", choices=["ratel", "reference"])
@@ -834,7 +942,11 @@ def main():
                     help="test mode: N ranks may share one GPU; gloo process group, library without NCCL")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--oracle-sample", type=int, default=1 << 25)
+    ap.add_argument("--oracle-sample", type=int, default=314_639_360,
+                    help="params per oracle pass (reference arm and cpu_baseline); default one whole 13B block")
+    ap.add_argument("--share-gpu", action="store_true",
+                    help="test mode: every rank on cuda:0 with real NCCL (each rank its own NCCL host id, "
+                         "loopback sockets); numbers are plumbing, not a scaling result")
     ap.add_argument("--overlap-tokens", type=int, default=8192, help="0 disables the AGO overlap probe")
     ap.add_argument("--overlap-host-tokens", type=int, default=131072,
                     help="pinned-host per-tensor AGO overlap probe (0 disables)")
@@ -852,28 +964,23 @@ def main():
     args = ap.parse_args()
     global ARM_AFTER
     ARM_AFTER = args.arm == "after"
-
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.steps < 1 or args.warmup < 0:
         raise SystemExit("need --steps >= 1")
+    world = relaunch_or_world(args)
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
 
     if args.impl == "reference":
-        if world > 1:
-            import torch.distributed as dist
-            dist.init_process_group("gloo")
         run_reference(args, rank, world)
-        if world > 1:
-            import torch.distributed as dist
-            dist.destroy_process_group()
         return
+    if args.share_gpu and world > 1:
+        share_gpu_nccl_env(rank)
 
     import torch
     import paper_conf_icde_liaosyxcyww25_b200 as R
     global SIM_COMM_NONE
     SIM_COMM_NONE = args.sim_comm_none
-    if SIM_COMM_NONE:
+    if SIM_COMM_NONE or args.share_gpu:
         local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device(f"cuda:{local}")
@@ -1036,15 +1143,17 @@ def main():
 
         cpu = None
         if rank == 0 and world == 1 and not args.no_cpu_baseline:
-            n = args.oracle_sample
+            # the oracle as it stands on this host: a whole 13B block per pass at
+            # every core (>= 8 s), and one pass of the same block on one core
             threads = host_threads()
-            v, done, dt = oracle_sample_rate(n, 2, threads, min_seconds=8.0)
-            v1, done1, dt1 = oracle_sample_rate(n // 8, 2, 1, min_seconds=3.0)
-            cpu = {"value": v, "unit": UNIT, "cores": threads, "kind": "oracle",
-                   "sample": f"{n:,} params (slice of block 0), {done} steps in {dt:.1f} s, "
-                             f"OpenMP {threads} threads",
-                   "single_thread": {"value": v1, "unit": UNIT, "cores": 1,
-                                     "sample": f"{n // 8:,} params, {done1} steps in {dt1:.1f} s"}}
+            n = args.oracle_sample
+            try:
+                cpu = oracle_baseline(n, 2, 1, threads, min_seconds=8.0)
+                one = oracle_baseline(n, 1, 0 if n >= (1 << 27) else 1, 1)
+                cpu["single_thread"] = {k: one[k] for k in ("value", "unit", "cores", "sample",
+                                                            "sample_ms_per_pass", "dram_gbs_at_28B_per_param")}
+            except Exception as ex:  # report, do not hide
+                cpu = {"value": None, "unit": UNIT, "cores": threads, "kind": "oracle", "error": repr(ex)[:300]}
 
         if rank == 0:
             line = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,

@@ -55,3 +55,50 @@ def test_reference_arm_under_torchrun_prints_once():
     lines = _lines(r.stdout)
     assert len(lines) == 1, r.stdout
     _check(lines[0], 2)
+
+
+def test_gpus_flag_relaunches_under_torchrun():
+    """`bench.py --gpus 2` outside torchrun re-launches itself with 2 ranks
+    (the flag was parsed and ignored, so an 8-GPU run would
+    have measured one GPU)."""
+    env = _env()
+    for k in ("WORLD_SIZE", "RANK", "LOCAL_RANK"):
+        env.pop(k, None)
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "2", "--steps", "1",
+                        "--warmup", "1", "--oracle-sample", "65536"], cwd=ROOT, capture_output=True, text=True,
+                       timeout=300, env=env)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = _lines(r.stdout)
+    assert len(lines) == 1, r.stdout
+    _check(lines[0], 2)
+    assert lines[0]["config"]["parallelism"].startswith("range-sharded x2")
+
+
+def test_world_size_mismatch_is_refused():
+    env = dict(_env(), WORLD_SIZE="2", RANK="0", LOCAL_RANK="0")
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--gpus", "4", "--steps", "1",
+                        "--oracle-sample", "65536"], cwd=ROOT, capture_output=True, text=True, timeout=120, env=env)
+    assert r.returncode == 2 and not _lines(r.stdout), (r.returncode, r.stdout)
+    assert "WORLD_SIZE=2" in r.stderr
+
+
+def test_reference_arm_reports_the_sample_it_timed():
+    """ms_per_step x steps must be time that actually ran (the driver's
+    consistency check): the step is one pass over the sample, with the host
+    facts and the implied DRAM rate in cpu_baseline."""
+    import time
+    t0 = time.time()
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--steps", "3", "--warmup", "1",
+                        "--oracle-sample", "200000"], cwd=ROOT, capture_output=True, text=True, timeout=300,
+                       env=_env())
+    wall = time.time() - t0
+    assert r.returncode == 0, r.stderr[-2000:]
+    (line,) = _lines(r.stdout)
+    assert line["steps"] * line["ms_per_step"] / 1e3 <= wall
+    cb = line["cpu_baseline"]
+    assert cb["sample_params"] == 200000 and cb["sample_passes"] == line["steps"]
+    assert abs(line["value"] - 200000 / (line["ms_per_step"] / 1e3)) <= 1e-6 * line["value"]
+    assert abs(cb["dram_gbs_at_28B_per_param"] - 28 * line["value"] / 1e9) <= 1e-9 * cb["dram_gbs_at_28B_per_param"]
+    for k in ("cpu_model", "numa_nodes", "sockets"):
+        assert k in cb
+    assert line["full_workload_ms_per_step_extrapolated"] > line["ms_per_step"]
