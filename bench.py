@@ -277,7 +277,11 @@ def workload_config(args, world):
                         f"per-block AGO hand-off" + (", clip" if args.clip > 0 else ""),
             "params": P, "blocks": len(sizes), "block_params": sizes[0], "residency": resid,
             "parallelism": (f"range-sharded x{world}" + (" (fused peer-store all-gather)" if args.fused_allgather else
-                                                          " (NCCL all-gather)")) if world > 1 else "single GPU",
+                                                          " (NCCL all-gather)")
+                            + (" [test mode: all ranks on cuda:0, NCCL over loopback sockets]" if args.share_gpu
+                               else "")
+                            + (" [test mode: all ranks on one GPU, no NCCL, P16 slices not exchanged]"
+                               if args.sim_comm_none else "")) if world > 1 else "single GPU",
             "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
             "max_grad_norm": args.clip, "update_streams": args.update_streams, "cta_tiles": args.cta_tiles,
             "k1_kernel": ["tma", "ldg", "ldg_lite"][args.k1_kernel], "staging": args.staging}
@@ -374,17 +378,21 @@ def linears(h):
 class SynthBackward:
     """Synthetic backward for the overlap measurement (harness, cuBLAS via
     torch): per block the dX and dW GEMMs of its four linears (4*P_blk*T
-    FLOPs), dW written into the block's grad-ring slot."""
-    def __init__(self, dev, h, tokens, p16_views, grad_ring, vocab_rows):
+    FLOPs), dW written into the block's grad-ring slot.  `chunk`: at most this
+    many tokens per GEMM (dW accumulated over chunks, like micro-batches), so
+    large T fits beside 13B device-resident states; None = one chunk."""
+    def __init__(self, dev, h, tokens, p16_views, grad_ring, vocab_rows, chunk=None):
         import torch
         self.h, self.T = h, tokens
+        self.C = min(tokens, chunk) if chunk else tokens
         self.dev = dev
         g = torch.Generator(device=dev)
         g.manual_seed(1)
         mk = lambda *s: (torch.randn(*s, device=dev, dtype=torch.bfloat16, generator=g) * 0.01)
-        self.X = {1: mk(tokens, h), 4: mk(tokens, 4 * h)}
-        self.dY = {3: mk(tokens, 3 * h), 1: mk(tokens, h), 4: mk(tokens, 4 * h)}
-        self.dX = torch.empty(tokens, 4 * h, device=dev, dtype=torch.bfloat16)
+        C = self.C
+        self.X = {1: mk(C, h), 4: mk(C, 4 * h)}
+        self.dY = {3: mk(C, 3 * h), 1: mk(C, h), 4: mk(C, 4 * h)}
+        self.dX = torch.empty(C, 4 * h, device=dev, dtype=torch.bfloat16)
         self.p16 = p16_views
         self.ring = grad_ring
         self.vocab_rows = vocab_rows
@@ -395,7 +403,7 @@ class SynthBackward:
         The linears run in backward order (fc2, fc1, proj, qkv); on_linear(j)
         is called after linear j's dW (per-tensor hand-off)."""
         import torch
-        h, T = self.h, self.T
+        h, T, C = self.h, self.T, self.C
         P = self.p16[b]
         G = self.ring[slot]
         if b == len(self.p16) - 1 and self.vocab_rows:
@@ -407,7 +415,11 @@ class SynthBackward:
             out.zero_()
             for t0 in range(0, T, 2048):
                 t1 = min(T, t0 + 2048)
-                out.addmm_(self.dYv[:t1 - t0].t(), X[t0:t1])
+                c0 = t0 % C
+                c1 = c0 + (t1 - t0)
+                if c1 > C:
+                    c0, c1 = 0, t1 - t0
+                out.addmm_(self.dYv[:t1 - t0].t(), X[c0:c1])
             return
         offs, off = [], 0
         for (o, i) in linears(h):
@@ -418,10 +430,63 @@ class SynthBackward:
             W = P[off:off + o * i].view(o, i)
             X = self.X[i // h]
             dY = self.dY[o // h]
-            torch.mm(dY, W, out=self.dX[:, :i])                          # dX = dY W
-            torch.mm(dY.t(), X, out=G[off:off + o * i].view(o, i))         # dW = dY^T X
+            dW = G[off:off + o * i].view(o, i)
+            for t0 in range(0, T, C):
+                c = min(C, T - t0)
+                torch.mm(dY[:c], W, out=self.dX[:c, :i])                    # dX = dY W
+                if t0 == 0:
+                    torch.mm(dY[:c].t(), X[:c], out=dW)                      # dW = dY^T X
+                else:
+                    dW.addmm_(dY[:c].t(), X[:c])                             # dW += dY^T X (next chunk)
             if on_linear is not None:
                 on_linear(j)
+
+
+class Energy:
+    """GPU energy counter (NVML total energy, mJ) of the bench's device."""
+
+    def __init__(self, uuid):
+        self.h = None
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByUUID(uuid)
+            self.nv.nvmlDeviceGetTotalEnergyConsumption(self.h)
+        except Exception:
+            self.h = None
+
+    def joules(self):
+        if self.h is None:
+            return None
+        return self.nv.nvmlDeviceGetTotalEnergyConsumption(self.h) / 1e3
+
+
+def _med(xs):
+    xs = sorted(x for x in xs if x is not None)
+    if not xs:
+        return None
+    k = len(xs)
+    return xs[k // 2] if k % 2 else 0.5 * (xs[k // 2 - 1] + xs[k // 2])
+
+
+def _spread(xs):
+    xs = [x for x in xs if x is not None]
+    return [min(xs), max(xs)] if xs else None
+
+
+def timed_run(torch, s, fn, energy=None):
+    """One run of fn on stream s: (CUDA-event ms on s, joules or None)."""
+    torch.cuda.synchronize()
+    j0 = energy.joules() if energy else None
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(s)
+    fn()
+    e1.record(s)
+    e1.synchronize()
+    torch.cuda.synchronize()
+    j1 = energy.joules() if energy else None
+    return e0.elapsed_time(e1), (j1 - j0 if j0 is not None and j1 is not None else None)
 
 
 SIM_COMM_NONE = False   # --sim-comm-none: N ranks on ONE GPU, gloo group, no NCCL (test mode)
@@ -454,64 +519,97 @@ def step_once(R, t, order, stream):
     R.ratel_sync(stream)
 
 
-def overlap_probe(args, R, torch, dev, model, sizes, order, t0):
-    """AGO overlapped with a synthetic backward of `args.overlap_tokens`
-    tokens vs the backward alone (Fig. 7 analog)."""
+def overlap_probe(args, R, torch, dev, model, sizes, order, t0, opt_ms, energy=None):
+    """C2 batch sweep (the Fig. 7 analog): for
+    each token count T the synthetic backward of the whole model alone, the
+    AGO step (armed first, every block's update enqueued at its hand-off,
+    grad ring recycled with ratel_block_wait) and the deferred "Ratel+ZeRO"
+    step (backward, then the whole optimizer step), alternated
+    `reps` times with the backward-alone baseline bracketing every repetition
+    (mean of the runs before and after).  Per run: CUDA-event time on the
+    backward stream and NVML energy.  Reported: medians and [min, max] over
+    repetitions of exposed optimizer ms, backward slowdown % and J per step."""
     L, h = SHAPES[args.shape]
     ring = model.grad_ring
     vocab = VOCAB if len(sizes) == L + 1 else 0
-    bw = SynthBackward(dev, h, args.overlap_tokens, model.p16, ring, vocab)
     s = torch.cuda.Stream(device=dev, priority=-2)
     nr = len(ring)
     t = [t0]
+    points = []
+    for T in args.overlap_sweep:
+        bw = SynthBackward(dev, h, T, model.p16, ring, vocab, chunk=16384)
 
-    def bwd_only():
-        with torch.cuda.stream(s):
-            for b in order:
-                bw.block(b, b % nr)
+        def bwd_only():
+            with torch.cuda.stream(s):
+                for b in order:
+                    bw.block(b, b % nr)
 
-    def ago():
-        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
-        t[0] += 1
-        with torch.cuda.stream(s):
-            for j, b in enumerate(order):
-                if j >= nr:
-                    R.ratel_block_wait(b + nr, s)       # ring slot consumed
-                bw.block(b, b % nr)
+        def arm():
+            R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+            t[0] += 1
+
+        def ago():
+            arm()
+            with torch.cuda.stream(s):
+                for j, b in enumerate(order):
+                    if j >= nr:
+                        R.ratel_block_wait(b + nr, s)       # ring slot consumed
+                    bw.block(b, b % nr)
+                    R.ratel_offload_grad_chunk(b, s)
+            R.ratel_sync(s)
+
+        def deferred():
+            bwd_only()
+            arm()
+            for b in order:                                  # every update after the whole backward
                 R.ratel_offload_grad_chunk(b, s)
-        R.ratel_sync(s)
+            R.ratel_sync(s)
 
-    res = {}
-    # the backward alone is timed before and after the AGO runs (the baseline
-    # drifts once the optimizer has run, see overlap_host_probe); mean used
-    for name, fn in (("bwd", bwd_only), ("ago", ago), ("bwd_after", bwd_only)):
-        fn()
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(s)
-        for _ in range(2):
-            fn()
-        e1.record(s)
-        e1.synchronize()
-        res[name] = e0.elapsed_time(e1) / 2
-    res["bwd_before_after"] = [res["bwd"], res["bwd_after"]]
-    res["bwd"] = 0.5 * (res["bwd"] + res["bwd_after"])
-    del bw
-    torch.cuda.empty_cache()
-    return res, t[0]
+        bwd_only()                                           # warm-up (cuBLAS heuristics, clocks)
+        ago()
+        runs = {"bwd": [timed_run(torch, s, bwd_only, energy)], "ago": [], "deferred": []}
+        for _ in range(args.overlap_reps):
+            runs["ago"].append(timed_run(torch, s, ago, energy))
+            runs["deferred"].append(timed_run(torch, s, deferred, energy))
+            runs["bwd"].append(timed_run(torch, s, bwd_only, energy))
+        base = [0.5 * (runs["bwd"][i][0] + runs["bwd"][i + 1][0]) for i in range(args.overlap_reps)]
+        ebase = [0.5 * (runs["bwd"][i][1] + runs["bwd"][i + 1][1]) if runs["bwd"][i][1] is not None else None
+                 for i in range(args.overlap_reps)]
+        pt = {"tokens": T, "reps": args.overlap_reps, "backward_ms": _med(base), "backward_ms_spread": _spread(base),
+              "backward_ms_runs": [r[0] for r in runs["bwd"]], "optimizer_alone_ms": opt_ms}
+        for k in ("ago", "deferred"):
+            exp = [runs[k][i][0] - base[i] for i in range(args.overlap_reps)]
+            pt[f"{k}_step_ms"] = _med([r[0] for r in runs[k]])
+            pt[f"{k}_exposed_ms"] = _med(exp)
+            pt[f"{k}_exposed_ms_spread"] = _spread(exp)
+            pt[f"{k}_backward_slowdown_pct"] = _med([100 * e / b for e, b in zip(exp, base)])
+            pt[f"{k}_hidden_fraction"] = _med([1 - e / opt_ms for e in exp])
+            if runs[k][0][1] is not None:
+                pt[f"{k}_joules_per_step"] = _med([r[1] for r in runs[k]])
+                pt[f"{k}_extra_joules_over_backward"] = _med([r[1] - e for r, e in zip(runs[k], ebase)])
+        if runs["bwd"][0][1] is not None:
+            pt["backward_joules"] = _med(ebase)
+        points.append(pt)
+        del bw
+        torch.cuda.empty_cache()
+    return points, t[0]
 
 
 HOST_ENQUEUE_MS = []   # host time to issue one step (arm + hand-offs + stream sync)
 
 
-def overlap_host_probe(args, R, torch, dev, dev_index):
+def overlap_host_probe(args, R, torch, dev, dev_index, energy=None):
     """The north star's host-resident overlap target (Fig. 7 analog): pinned-host
     states of `--overlap-host-blocks` 13B blocks, each of a block's four linears
     registered as its own unit and handed off right after its dW GEMM (the
-    paper's per-tensor hand-off), with a synthetic backward of
-    `--overlap-host-tokens` tokens.  Exposed = AGO step - backward alone.
+    paper's per-tensor hand-off), with a synthetic backward of T
+    tokens for every T of `--overlap-host-sweep`.  Per T: `reps` alternating
+    (AGO, backward-alone) runs after a backward-alone run, so every AGO run has
+    a baseline right before and right after it (their mean: the GPU's power
+    state drifts over the probe).  Exposed = AGO - baseline; hidden = 1 -
+    exposed / optimizer alone.  Medians and [min, max] over repetitions.
     Measured for the GPU-streamed residency (the north star's path) and, on the
-    same states and backward, for the paper's own CPU handler (HOST_COMPUTE).
+    same states and backward, the paper's own CPU handler (HOST_COMPUTE).
     Returns {residency: result}."""
     L, h = SHAPES[args.shape]
     sizes = model_blocks(args.shape, with_embedding=False)[:args.overlap_host_blocks]
@@ -529,19 +627,19 @@ def overlap_host_probe(args, R, torch, dev, dev_index):
         units.append([R.ratel_range(r0.param_bf16 + 2 * o, r0.grad_bf16 + 2 * o, 0, r0.master + 4 * o,
                                     r0.exp_avg + 4 * o, r0.exp_avg_sq + 4 * o, ln, 1) for o, ln in offs])
     K = 4
-    bw = SynthBackward(dev, h, args.overlap_host_tokens, model.p16, model.grad_ring, 0)
     s = torch.cuda.Stream(device=dev, priority=-2)
     order = list(reversed(range(len(sizes))))
     P = sum(sizes)
     out = {}
-    t_bwd = None
+    # one set of activations (<= 64K tokens per GEMM chunk) serves every T of the sweep
+    bw0 = SynthBackward(dev, h, max(args.overlap_host_sweep), model.p16, model.grad_ring, 0, chunk=65536)
     # settle the GPU at its thermal/power operating point first: measured, the same
     # backward runs ~10 % faster for the first several seconds of load
     w0 = time.time()
     while time.time() - w0 < 15.0:
         with torch.cuda.stream(s):
             for b in order:
-                bw.block(b, b % 3)
+                bw0.block(b, b % 3)
         torch.cuda.synchronize()
     try:
         for resname, code in (("pinned-host", R.RATEL_PINNED_HOST), ("hostcompute", R.RATEL_HOST_COMPUTE)):
@@ -552,11 +650,6 @@ def overlap_host_probe(args, R, torch, dev, dev_index):
                         R.ratel_register_block(b * K + j, [r], code)
                 t = [1]
 
-                def bwd():
-                    with torch.cuda.stream(s):
-                        for b in order:
-                            bw.block(b, b % 3)
-
                 def opt():
                     R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
                     t[0] += 1
@@ -565,48 +658,64 @@ def overlap_host_probe(args, R, torch, dev, dev_index):
                             R.ratel_offload_grad_chunk(b * K + j, s)
                     R.ratel_sync(s)
 
-                def ago():
-                    R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
-                    t[0] += 1
-                    with torch.cuda.stream(s):
-                        for jb, b in enumerate(order):
-                            if jb >= 3:
-                                for j in range(K):
-                                    R.ratel_block_wait((b + 3) * K + j, s)   # ring slot consumed
-                            bw.block(b, b % 3, on_linear=lambda j, b=b: R.ratel_offload_grad_chunk(b * K + j, s))
-                    R.ratel_sync(s)
+                opt()
+                opt_runs = [timed_run(torch, s, opt, energy) for _ in range(2)]
+                opt_ms = _med([r[0] for r in opt_runs])
+                pts = []
+                for T in args.overlap_host_sweep:
+                    bw = bw0
+                    bw.T = T
 
-                res = {}
-                # the backward alone is timed right before the optimizer and right after the
-                # AGO runs and averaged: a GPU settling at its power cap slows the same
-                # backward over the probe, and one early baseline would count that as exposure
-                for name, fn in (("bwd", bwd), ("opt", opt), ("ago", ago), ("bwd_after", bwd)):
-                    fn()
-                    torch.cuda.synchronize()
-                    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-                    e0.record(s)
-                    for _ in range(2):
-                        fn()
-                    e1.record(s)
-                    e1.synchronize()
-                    res[name] = e0.elapsed_time(e1) / 2
-                t_bwd = 0.5 * (res["bwd"] + res["bwd_after"])
-                r = {"tokens": args.overlap_host_tokens, "blocks": len(sizes), "params": P,
-                     "residency": resname, "handoff": "per tensor (4 linears per block)",
-                     "backward_ms": t_bwd, "backward_ms_before_after": [res["bwd"], res["bwd_after"]],
-                     "optimizer_alone_ms": res["opt"], "ago_step_ms": res["ago"],
-                     "exposed_optimizer_ms": res["ago"] - t_bwd,
-                     "hidden_fraction": 1.0 - (res["ago"] - t_bwd) / res["opt"],
-                     "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)"}
+                    def bwd():
+                        with torch.cuda.stream(s):
+                            for b in order:
+                                bw.block(b, b % 3)
+
+                    def ago():
+                        R.ratel_adam_step(HP["lr"], HP["beta1"], HP["beta2"], HP["eps"], HP["weight_decay"], t[0])
+                        t[0] += 1
+                        with torch.cuda.stream(s):
+                            for jb, b in enumerate(order):
+                                if jb >= 3:
+                                    for j in range(K):
+                                        R.ratel_block_wait((b + 3) * K + j, s)   # ring slot consumed
+                                bw.block(b, b % 3, on_linear=lambda j, b=b: R.ratel_offload_grad_chunk(b * K + j, s))
+                        R.ratel_sync(s)
+
+                    ago()                                    # warm-up at this T
+                    runs_b = [timed_run(torch, s, bwd, energy)]
+                    runs_a = []
+                    for _ in range(args.overlap_reps):
+                        runs_a.append(timed_run(torch, s, ago, energy))
+                        runs_b.append(timed_run(torch, s, bwd, energy))
+                    base = [0.5 * (runs_b[i][0] + runs_b[i + 1][0]) for i in range(args.overlap_reps)]
+                    exp = [a[0] - b for a, b in zip(runs_a, base)]
+                    hid = [1 - e / opt_ms for e in exp]
+                    pt = {"tokens": T, "reps": args.overlap_reps, "backward_ms": _med(base),
+                          "backward_ms_runs": [r[0] for r in runs_b], "ago_step_ms": _med([a[0] for a in runs_a]),
+                          "exposed_optimizer_ms": _med(exp), "exposed_ms_spread": _spread(exp),
+                          "hidden_fraction": _med(hid), "hidden_fraction_spread": _spread(hid)}
+                    if runs_a[0][1] is not None:
+                        eb = [0.5 * (runs_b[i][1] + runs_b[i + 1][1]) for i in range(args.overlap_reps)]
+                        pt["backward_joules"] = _med(eb)
+                        pt["ago_extra_joules_over_backward"] = _med([a[1] - e for a, e in zip(runs_a, eb)])
+                    pts.append(pt)
+                r = {"blocks": len(sizes), "params": P, "residency": resname,
+                     "handoff": "per tensor (4 linears per block)", "optimizer_alone_ms": opt_ms,
+                     "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)",
+                     "points": pts}
                 if code == R.RATEL_PINNED_HOST:
-                    r["host_link_gbs_optimizer_alone"] = 24 * P / (res["opt"] / 1e3) / 1e9
+                    r["host_link_gbs_optimizer_alone"] = 24 * P / (opt_ms / 1e3) / 1e9
                 else:
                     r["handler"] = "the paper's CPU AdamW (HOST_COMPUTE): G16 D2H, CPU update, P16 H2D"
+                if opt_runs[0][1] is not None:
+                    r["optimizer_alone_joules"] = _med([x[1] for x in opt_runs])
                 out[resname] = r
             finally:
                 R.ratel_finalize()
         return out
     finally:
+        del bw0
         del model
         torch.cuda.empty_cache()
 
@@ -642,6 +751,57 @@ def barrier(torch, world):
         import torch.distributed as dist
         dist.barrier()
     torch.cuda.synchronize()
+
+
+# ------------------------------------------------------------ N > 1 probes
+C3_SLICE_N8 = 77_081_984          # 30B block (616,655,872 params) / 8 ranks: SURVEY §8(a) C3
+
+
+def nccl_allgather_probe(torch, dev, world, counts, reps=5):
+    """NCCL bf16 all-gather bus bandwidth at the given per-rank counts
+    (torch.distributed on the same NCCL): busbw = (N-1)/N * N*count*2 B / t,
+    median of `reps` after one warm-up, CUDA events, max over ranks.  The
+    denominator of roofline.nvlink (SURVEY §8(d) roofline probe 4)."""
+    import torch.distributed as dist
+    out = {}
+    for name, c in counts.items():
+        send = torch.empty(c, dtype=torch.bfloat16, device=dev).fill_(1.0)
+        recv = torch.empty(c * world, dtype=torch.bfloat16, device=dev)
+        dist.all_gather_into_tensor(recv, send)
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(reps):
+            dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            dist.all_gather_into_tensor(recv, send)
+            e1.record()
+            e1.synchronize()
+            ts.append(max_over_ranks(torch, e0.elapsed_time(e1), world, dev))
+        t = sorted(ts)[len(ts) // 2]
+        out[name] = {"count_per_rank": c, "bytes_per_rank": 2 * c, "ms": t,
+                     "busbw_gbs": (world - 1) / world * world * 2 * c / (t / 1e3) / 1e9,
+                     "algbw_gbs": world * 2 * c / (t / 1e3) / 1e9}
+        del send, recv
+    torch.cuda.empty_cache()
+    return out
+
+
+def host_link_probe_all_ranks(torch, dev, world):
+    """The duplex host-link probe run in every rank at once (started behind a
+    barrier): per-rank and aggregate GB/s -- the pinned-host roofline at this
+    N, where ranks may share PCIe switches and host DRAM (SURVEY §8(d) probe 3)."""
+    import torch.distributed as dist
+    barrier(torch, world)
+    mine = host_link_probe(torch, dev)
+    vals = torch.tensor([mine["h2d"], mine["d2h"], mine["duplex"]], dtype=torch.float64,
+                        device=dev if dist.get_backend() == "nccl" else "cpu")
+    allv = [torch.zeros_like(vals) for _ in range(world)]
+    dist.all_gather(allv, vals)
+    per = [[float(x) for x in v.cpu()] for v in allv]
+    return {"per_rank": [{"h2d": a, "d2h": b, "duplex": c} for a, b, c in per],
+            "aggregate_duplex_gbs": sum(r[2] for r in per), "min_rank_duplex_gbs": min(r[2] for r in per),
+            "note": "every rank's pinned H2D || D2H probe concurrently"}
 
 
 # ------------------------------------------------------------------- e2e
@@ -947,9 +1107,13 @@ def main():
     ap.add_argument("--share-gpu", action="store_true",
                     help="test mode: every rank on cuda:0 with real NCCL (each rank its own NCCL host id, "
                          "loopback sockets); numbers are plumbing, not a scaling result")
-    ap.add_argument("--overlap-tokens", type=int, default=8192, help="0 disables the AGO overlap probe")
-    ap.add_argument("--overlap-host-tokens", type=int, default=131072,
-                    help="pinned-host per-tensor AGO overlap probe (0 disables)")
+    ap.add_argument("--overlap-sweep", type=lambda x: [int(v) for v in x.split(",") if v], default=[2048, 8192, 32768, 65536],
+                    help="device-resident AGO vs deferred overlap sweep: tokens per step, comma-separated "
+                         "('' disables)")
+    ap.add_argument("--overlap-reps", type=int, default=3, help="alternating repetitions per overlap point")
+    ap.add_argument("--overlap-host-sweep", type=lambda x: [int(v) for v in x.split(",") if v],
+                    default=[32768, 65536, 98304, 131072, 196608],
+                    help="pinned-host per-tensor AGO overlap probe: tokens per step, comma-separated ('' disables)")
     ap.add_argument("--overlap-host-blocks", type=int, default=8)
     ap.add_argument("--arm", default="before", choices=["before", "after"],
                     help="arm before the hand-offs (AGO) or after the last one (deferred)")
@@ -1092,18 +1256,44 @@ def main():
                                "loop splits work statically; K1 schedules tiles dynamically and can exceed it",
                 "ncu_dram_pct_of_peak": ncu_summary().get("ncu_dram_pct_of_peak_sustained")}
         overlap = None
-        if args.overlap_tokens > 0 and world == 1 and args.residency == "device" and args.clip == 0:
+        if args.overlap_sweep and world == 1 and args.residency == "device" and args.clip == 0:
             try:
-                o, t = overlap_probe(args, R, torch, dev, model, sizes, order, t)
-                opt_ms = ms / args.steps
-                overlap = {"tokens": args.overlap_tokens, "backward_ms": o["bwd"],
-                           "backward_ms_before_after": o["bwd_before_after"], "ago_step_ms": o["ago"],
-                           "optimizer_alone_ms": opt_ms, "exposed_optimizer_ms": o["ago"] - o["bwd"],
-                           "hidden_fraction": 1.0 - (o["ago"] - o["bwd"]) / opt_ms,
-                           "backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16)",
-                           "grad_ring": len(model.grad_ring)}
+                pts, t = overlap_probe(args, R, torch, dev, model, sizes, order, t, ms / args.steps,
+                                       Energy(gpu_uuid(torch, dev)))
+                overlap = {"backward": "synthetic: dX and dW GEMMs of each block's 4 linears (cuBLAS bf16), "
+                                       "<= 16K tokens per GEMM chunk", "grad_ring": len(model.grad_ring),
+                           "schedules": "ago = armed before backward, per-block hand-off; deferred = whole "
+                                        "backward, then the whole step (Ratel+ZeRO)",
+                           "energy": "NVML total-energy counter around each run", "points": pts}
             except Exception as ex:
                 overlap = {"error": repr(ex)[:300]}
+        multi = None
+        if world > 1 and not SIM_COMM_NONE:
+            try:
+                own_max = max(e - b for (b, e) in model.slices)
+                probes = nccl_allgather_probe(torch, dev, world, {
+                    "c3_block_slice_n8": C3_SLICE_N8,
+                    "this_workload_block_slice": R.ratel_padded_numel(max(sizes), world) // world})
+                bw = probes["this_workload_block_slice"]["busbw_gbs"]
+                nv_bytes = 2.0 * (world - 1) / world * P          # bf16 P16 received per GPU per step
+                step_s = ms / args.steps / 1e3
+                t_hbm = BYTES_PER_PARAM * (P / world) / (peak * 1e9)
+                t_nv = nv_bytes / (bw * 1e9)
+                roof["nvlink"] = {"bound": "nvlink", "collective": "per-block bf16 all-gather (X2)",
+                                  "algorithmic_bytes_per_gpu_per_step": nv_bytes,
+                                  "achieved": nv_bytes / step_s / 1e9, "peak": bw, "unit": "GB/s",
+                                  "frac": nv_bytes / step_s / 1e9 / bw,
+                                  "peak_source": "this run's NCCL all-gather busbw at the workload's per-rank "
+                                                 "block slice", "spec_gbs_per_direction": 900.0}
+                roof["step_bounds_ms"] = {"hbm": 1e3 * t_hbm, "nvlink": 1e3 * t_nv,
+                                          "max": 1e3 * max(t_hbm, t_nv),
+                                          "step_over_max_bound": (ms / args.steps) / (1e3 * max(t_hbm, t_nv))}
+                multi = {"nccl_allgather": probes, "host_link": host_link_probe_all_ranks(torch, dev, world),
+                         "own_params_max_rank": own_max,
+                         "transport": ("loopback sockets, all ranks on one GPU (--share-gpu test mode)"
+                                       if args.share_gpu else "NCCL over NVLink/NVSwitch")}
+            except Exception as ex:  # report, do not hide
+                multi = {"error": repr(ex)[:300]}
         e2e = None
         if not args.no_e2e and args.residency == "device":
             try:
@@ -1133,9 +1323,9 @@ def main():
                 roof = dict(roof, offdevice_error=repr(ex)[:300])
 
         overlap_host = overlap_hostcompute = None
-        if args.overlap_host_tokens > 0 and world == 1 and args.residency == "device":
+        if args.overlap_host_sweep and world == 1 and args.residency == "device":
             try:
-                oh = overlap_host_probe(args, R, torch, dev, local)
+                oh = overlap_host_probe(args, R, torch, dev, local, Energy(gpu_uuid(torch, dev)))
                 overlap_host, overlap_hostcompute = oh.get("pinned-host"), oh.get("hostcompute")
             except Exception as ex:  # report, do not hide
                 overlap_host = {"error": repr(ex)[:300]}
@@ -1167,6 +1357,8 @@ def main():
                     "host_enqueue_ms_first_step": HOST_ENQUEUE_MS[0] if HOST_ENQUEUE_MS else None,
                     "overlap": overlap, "overlap_host": overlap_host, "overlap_hostcompute": overlap_hostcompute,
                     "hbm_gbs_step": BYTES_PER_PARAM * P / (ms / args.steps / 1e3) / 1e9 / world}
+            if multi is not None:
+                line["multi_gpu"] = multi
             print(json.dumps(line), flush=True)
     finally:
         try:

@@ -229,9 +229,14 @@ int ratel_register_block(int block_id, const ratel_range* ranges, int n_ranges, 
  * NULL entries are skipped.  From then on the update kernel stores this
  * rank's P16 slice of that range directly into every peer's buffer (NVLink
  * P2P stores inside the kernel, overlapping the HBM streaming) and the NCCL
- * all-gather of that range is skipped; ratel_sync adds one 8-byte allreduce
- * as the cross-rank barrier.  Not for RATEL_HOST_COMPUTE blocks.  Between
- * steps only.  The pointers are borrowed like all registered memory. */
+ * all-gather of that range is skipped.  Synchronisation (NCCL communicator
+ * present): each hand-off of such a block adds an 8-byte allreduce on the
+ * comm stream and the block's update waits for it -- every rank has handed
+ * the block off, so no rank's backward still reads the P16 the peers are
+ * about to overwrite -- and ratel_sync adds one more as the "all peer stores
+ * landed" barrier.  With RATEL_COMM_NONE the caller provides that ordering.
+ * Not for RATEL_HOST_COMPUTE blocks.  Between steps only.  The pointers are
+ * borrowed like all registered memory. */
 int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_params, int n);
 
 /* Fused data-parallel gradient reduction (reduce-scatter folded into the
@@ -297,7 +302,11 @@ int ratel_offload_grad_chunk(int block_id, void* stream);
  * memory side of active gradient offloading: a block's G16 is dead as soon as
  * its handler ran.  RATEL_ESTATE if the block was handed off
  * in the current step but its update is not enqueued yet (deferred mode) or
- * it is not registered. */
+ * it is not registered.  RATEL_SSD blocks: the library's reader thread issues
+ * the block's grad reads on its own streams, so until ratel_block_wait (which
+ * waits on the host until the reader has issued them, then orders `stream` and
+ * the optimizer stream after them) or ratel_sync, record_stream on the
+ * optimizer stream does not cover them -- keep the grad alive until then. */
 int ratel_block_wait(int block_id, void* stream);
 
 /* Ends the step: `stream` (cudaStream_t) is ordered after every update,
@@ -324,6 +333,21 @@ uint64_t ratel_padded_numel(uint64_t numel, int world_size);
  * s = ratel_padded_numel(numel, N)/N, begin = min(numel, rank*s),
  * end = min(numel, begin + s).  Pure host function. */
 int ratel_rank_slice(uint64_t numel, int world_size, int rank, uint64_t* begin, uint64_t* end);
+
+/* Rebuilds block `block_id`'s working copy from its master weights:
+ * P16[slice] = bf16_rne(master) for this rank's slice of every range (the
+ * same RNE conversion the update uses, "produces a 16-bit
+ * parameter copy"), then -- N > 1 -- the bf16 all-gather (NCCL in place, or
+ * the peer stores of ratel_register_peer_params plus an 8-byte barrier), so
+ * every rank's full P16 matches the restored masters.  For checkpoint resume
+ * (restore master/m/v, then call this for every block) or any out-of-band
+ * change of the masters.  Ordered after the work already on `stream`
+ * (cudaStream_t); `stream` is ordered after the refresh (NULL: the host
+ * blocks until done).  Device, pinned-host and HOST_COMPUTE masters are read
+ * in place; RATEL_SSD masters are read from the state file (the calling
+ * thread preads tile by tile).  Between steps only (RATEL_ESTATE otherwise);
+ * collective when world_size > 1 (every rank, same blocks, same order). */
+int ratel_refresh_params(int block_id, void* stream);
 
 /* The optimizer stream (cudaStream_t) -- for torch's record_stream. NULL before init. */
 void* ratel_optimizer_stream(void);

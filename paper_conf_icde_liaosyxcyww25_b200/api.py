@@ -82,14 +82,49 @@ class _SsdFile:
         self.fd = self.fd_buf = None
 
 
+class _SymmArena:
+    """Data-parallel buffers for world > 1: every range's P16 and G16 carved
+    out of two flat torch symmetric-memory allocations (one rendezvous each),
+    so every rank can map every other rank's buffers -- the peer pointers the
+    fused reduce-scatter (ratel_register_peer_grads) and the fused all-gather
+    (ratel_register_peer_params) need."""
+
+    def __init__(self, caps, dev):
+        import torch.distributed as dist
+        import torch.distributed._symmetric_memory as symm_mem
+        self.offs, off = [], 0
+        for c in caps:
+            self.offs.append(off)
+            off += (c + 7) // 8 * 8          # 16-byte aligned views
+        self.p16 = symm_mem.empty(max(off, 8), dtype=torch.bfloat16, device=dev)
+        self.g16 = symm_mem.empty(max(off, 8), dtype=torch.bfloat16, device=dev)
+        self.p16.zero_()
+        self.g16.zero_()
+        group = dist.group.WORLD.group_name
+        self.hp = symm_mem.rendezvous(self.p16, group)
+        self.hg = symm_mem.rendezvous(self.g16, group)
+        self.next = 0
+
+    def take(self, cap):
+        k = self.next
+        self.next += 1
+        o = self.offs[k]
+        return (self.p16[o:o + cap], self.g16[o:o + cap],
+                [b + 2 * o for b in self.hp.buffer_ptrs], [b + 2 * o for b in self.hg.buffer_ptrs])
+
+
 class _Range:
-    def __init__(self, params, apply_wd, world, rank, dev, residency, ssd=None):
+    def __init__(self, params, apply_wd, world, rank, dev, residency, ssd=None, arena=None):
         self.params = params
         self.numel = sum(p.numel() for p in params)
         cap = R.ratel_padded_numel(self.numel, world)
         beg, end = R.ratel_rank_slice(self.numel, world, rank)
-        self.p16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
-        self.g16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+        self.peer_p16 = self.peer_g16 = None
+        if arena is not None:   # world > 1, data parallel: symmetric memory
+            self.p16, self.g16, self.peer_p16, self.peer_g16 = arena.take(cap)
+        else:
+            self.p16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+            self.g16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
         flat32 = torch.cat([p.detach().reshape(-1).to(torch.float32) for p in params]).to(dev)
         s = max(end - beg, 8)
         self.ssd, self.ssd_off = ssd, None
@@ -181,11 +216,23 @@ class Ratel_Optimizer:
     handler.  Finer units shorten the update tail after the
     last gradient (a block's update done 12-13 ms after its last gradient instead
     of ~70 ms, profiles/r01_overlap_granularity.jsonl); the result is bitwise the same.
-    `blocks`/`block_ids`/`state(i)` then index units."""
+    `blocks`/`block_ids`/`state(i)` then index units.
+
+    Data parallelism (torch.distributed initialised, world > 1; one process
+    per GPU): every rank runs its own micro-batch and each hook hands off the
+    rank's LOCAL gradient.  data_parallel="fused" (default) allocates P16 and
+    G16 in torch symmetric memory and registers every rank's buffers with the
+    library, so each rank's update kernel reduces the N local gradients of its
+    slice (mean, fp64, R17) and stores its P16 slice into every
+    rank's copy (fused reduce-scatter + all-gather over NVLink; residency
+    "device" or "host").  data_parallel="reduced" is for callers whose
+    gradients are already identical on every rank when the hook fires (the
+    library then only all-gathers P16 over NCCL, R11).  Both sides of a step
+    are collective: every rank hands off the same units in the same order."""
 
     def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,
                  residency="device", no_decay=None, first_block_id=0, granularity="block", ssd_path=None,
-                 hybrid_gpu_frac=0.3):
+                 hybrid_gpu_frac=0.3, data_parallel="fused"):
         import torch.distributed as dist
         distributed = dist.is_available() and dist.is_initialized()
         world = dist.get_world_size() if distributed else 1
@@ -213,13 +260,23 @@ class Ratel_Optimizer:
                     units.append([(nodecay, False)])
         if residency == "hybrid" and world > 1:
             raise ValueError('residency="hybrid" is single-rank')
+        if data_parallel not in ("fused", "reduced"):
+            raise ValueError(f"data_parallel must be 'fused' or 'reduced', not {data_parallel!r}")
+        fused_dp = world > 1 and data_parallel == "fused"
+        if fused_dp and residency not in ("device", "host"):
+            raise ValueError(f'data_parallel="fused" needs residency "device" or "host", not {residency!r} '
+                             f'(the fused reduction reads peer gradients inside the update kernel)')
+        arena = None
+        if fused_dp:
+            caps = [R.ratel_padded_numel(sum(p.numel() for p in ps), world) for groups in units for ps, _ in groups]
+            arena = _SymmArena(caps, dev)
         ssd = residency in ("ssd", "ssd_hostcompute")
         if ssd and not ssd_path:
             raise ValueError(f'residency="{residency}" needs ssd_path (the state file to create)')
         self.ssd = _SsdFile(ssd_path) if ssd else None
         for j, groups in enumerate(units):
-            ranges = [_Range(ps, wd, world, rank, dev, "host" if residency == "hybrid" else residency, self.ssd)
-                      for ps, wd in groups]
+            ranges = [_Range(ps, wd, world, rank, dev, "host" if residency == "hybrid" else residency, self.ssd,
+                             arena) for ps, wd in groups]
             self.blocks.append(ranges)
             self.block_ids.append(first_block_id + j)
         if self.ssd is not None:
@@ -246,6 +303,10 @@ class Ratel_Optimizer:
             if self.ssd is not None:
                 for i, r in enumerate(ranges):
                     R.ratel_register_ssd(bid, i, self.ssd.fd, r.ssd_off)
+            if fused_dp:
+                for i, r in enumerate(ranges):
+                    R.ratel_register_peer_grads(bid, i, r.peer_g16, 1.0 / world)
+                    R.ratel_register_peer_params(bid, i, r.peer_p16)
         self._pending = {}
         self._handed = set()
         self._hooks = []
@@ -319,17 +380,21 @@ class Ratel_Optimizer:
                 "weight_decay": self.weight_decay, "ranges": out}
 
     def load_state_dict(self, sd: dict) -> None:
-        """Restore states saved by state_dict() (same block/range layout) and
-        refresh P16 = bf16(master) through the library on the next step; the
-        step counter continues from sd["t"].  Call between steps."""
+        """Restore states saved by state_dict() (same block/range layout; this
+        rank's slices) and rebuild the model's P16 from the restored masters in
+        the library (ratel_refresh_params: bf16 RNE of the rank slice, then the
+        all-gather across ranks); the step counter continues from sd["t"].
+        Call between steps, on every rank."""
         assert len(sd["ranges"]) == len(self.blocks)
         for ranges, saved in zip(self.blocks, sd["ranges"]):
             assert len(ranges) == len(saved)
             for r, s in zip(ranges, saved):
                 r.load_states(s["master"], s["exp_avg"], s["exp_avg_sq"])
-                beg, end = r.slice
-                if end > beg:  # the model's working copy must match the restored master
-                    r.p16[beg:end].copy_(s["master"][:end - beg].to(r.p16.device).to(torch.bfloat16))
+        torch.cuda.synchronize()   # pinned-host / file states written before the library reads them
+        s = torch.cuda.current_stream()
+        for bid in self.block_ids:
+            for lid in self._lib_ids[bid]:
+                R.ratel_refresh_params(lid, s)
         self.t = int(sd["t"])
         self.lr, self.betas, self.eps, self.weight_decay = sd["lr"], tuple(sd["betas"]), sd["eps"], sd["weight_decay"]
         torch.cuda.synchronize()

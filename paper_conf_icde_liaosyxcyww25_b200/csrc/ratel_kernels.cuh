@@ -1018,6 +1018,35 @@ __global__ void __launch_bounds__(kThreads) grad_sumsq_rs_kernel(const __grid_co
   if (threadIdx.x == 0) P.partials[blockIdx.x] = t;
 }
 
+// P16 refresh (ratel_refresh_params): p = bf16_rne(theta) over a rank slice,
+// with the same cvt.rn.bf16x2.f32 as K1's P16 store, also into every peer's
+// buffer (fused all-gather).  theta may be device memory or page-locked host
+// memory read in place over the link (unified addressing); 16-byte vectors.
+__global__ void __launch_bounds__(kThreads) refresh_p16_kernel(const float* __restrict__ th, uint16_t* __restrict__ p,
+                                                               uint64_t n, const __grid_constant__ PeerDesc pd) {
+  const uint64_t tid = static_cast<uint64_t>(blockIdx.x) * blockDim.x + threadIdx.x;
+  const uint64_t stride = static_cast<uint64_t>(gridDim.x) * blockDim.x;
+  const uint64_t n8 = n >> 3;
+  for (uint64_t i = tid; i < n8; i += stride) {
+    const float4 a = *reinterpret_cast<const float4*>(th + 8 * i);
+    const float4 b = *(reinterpret_cast<const float4*>(th + 8 * i) + 1);
+    uint4 pk;
+    pk.x = pack_bf16x2_rn(a.x, a.y);
+    pk.y = pack_bf16x2_rn(a.z, a.w);
+    pk.z = pack_bf16x2_rn(b.x, b.y);
+    pk.w = pack_bf16x2_rn(b.z, b.w);
+    *reinterpret_cast<uint4*>(p + 8 * i) = pk;
+    st_peers8(pd, 8 * i, pk);
+  }
+  const uint64_t j = (n8 << 3) + tid;
+  if (j < n) {
+    const uint16_t pb = static_cast<uint16_t>(pack_bf16x2_rn(th[j], 0.0f) & 0xFFFFu);
+    p[j] = pb;
+    for (int q = 0; q < pd.n; ++q) pd.p[q][j] = pb;
+  }
+  if (pd.n > 0) __threadfence_system();
+}
+
 // K3.  One CTA sums `count` partial slots in a fixed order into *out.
 __global__ void __launch_bounds__(kThreads) sumsq_finalize_kernel(const double* __restrict__ partials,
                                                                  uint64_t count, double* out) {

@@ -90,7 +90,10 @@ struct Block {
   std::vector<std::vector<const uint16_t*>> rgrads;
   std::vector<double> rscale;
   bool rs = false;                  // some range of this block has peer grads
-  cudaEvent_t ev_ready = nullptr;   // RS + NCCL: every rank's G16 of this block is complete
+  bool pp = false;                  // some range of this block has peer params (fused all-gather)
+  // RS or PP + NCCL: every rank has handed this block off -- its G16 is complete
+  // everywhere, and no rank's backward still reads the P16 the peers will overwrite
+  cudaEvent_t ev_ready = nullptr;
   cudaEvent_t ev_rel = nullptr;     // RS + NCCL: every rank finished reading this block's G16
   bool handed_off = false, enqueued = false;
   // SSD residency: per range, the state file and where the slice's arrays are
@@ -123,6 +126,7 @@ struct SsdEngine {
   std::deque<SsdTile> wq;
   int slot_busy[kMaxDepth] = {};  // a tile in this slot still awaits its write-back
   bool stop = false;
+  bool reader_done = false;  // the writer drains until the reader can queue no more tiles
   uint64_t jobs_in = 0, jobs_out = 0, tiles_in = 0, tiles_out = 0;
   int err = 0;
   std::string msg;
@@ -891,7 +895,12 @@ void ssd_reader_main(SsdEngine* E) {
     {
       std::unique_lock<std::mutex> lk(E->mu);
       E->cv.wait(lk, [&] { return E->stop || !E->jobs.empty(); });
-      if (E->jobs.empty()) return;  // stop
+      if (E->jobs.empty()) {  // stop
+        E->reader_done = true;
+        lk.unlock();
+        E->cv.notify_all();
+        return;
+      }
       job = E->jobs.front();
       E->jobs.pop_front();
     }
@@ -921,7 +930,9 @@ void ssd_writer_main(SsdEngine* E) {
     bool failed;
     {
       std::unique_lock<std::mutex> lk(E->mu);
-      E->cv.wait(lk, [&] { return E->stop || !E->wq.empty(); });
+      // exit only once the reader has stopped: a job still in flight may be
+      // waiting for a ring slot that only this thread's write-back frees
+      E->cv.wait(lk, [&] { return (E->stop && E->reader_done) || !E->wq.empty(); });
       if (E->wq.empty()) return;  // stop
       t = E->wq.front();
       E->wq.pop_front();
@@ -1050,7 +1061,7 @@ int enqueue_block(Block& B, const std::vector<cudaEvent_t>* ssd_wait = nullptr) 
     if (G.cfg.update_streams > 1) {
       ks = G.s_k[G.k_next++ & 1u];
       CK(cudaStreamWaitEvent(ks, B.ev_grad, 0));
-      if (B.rs && G.comm != nullptr) CK(cudaStreamWaitEvent(ks, B.ev_ready, 0));
+      if ((B.rs || B.pp) && G.comm != nullptr) CK(cudaStreamWaitEvent(ks, B.ev_ready, 0));
       if (G.cfg.max_grad_norm > 0.0) CK(cudaStreamWaitEvent(ks, G.ev_norm, 0));
     }
     RangeDesc rd[kMaxRanges];
@@ -1078,7 +1089,7 @@ int enqueue_block(Block& B, const std::vector<cudaEvent_t>* ssd_wait = nullptr) 
     // Tile updates run on a HIGH-priority stream: each is short and gates the
     // copy pipeline, so when a backward GEMM frees SMs they must go first.
     CK(cudaStreamWaitEvent(G.s_tile, B.ev_grad, 0));
-    if (B.rs && G.comm != nullptr) CK(cudaStreamWaitEvent(G.s_tile, B.ev_ready, 0));
+    if ((B.rs || B.pp) && G.comm != nullptr) CK(cudaStreamWaitEvent(G.s_tile, B.ev_ready, 0));
     if (G.cfg.max_grad_norm > 0.0) CK(cudaStreamWaitEvent(G.s_tile, G.ev_norm, 0));
     for (size_t i = 0; i < B.ranges.size(); ++i) {
       const Slice& s = B.slices[i];
@@ -1500,9 +1511,14 @@ int ratel_register_peer_params(int block_id, int range_idx, void* const* peer_pa
       return set_error(RATEL_EINVAL, "ratel_register_peer_params: peer pointers must be 16-byte aligned");
     v[q] = static_cast<uint16_t*>(peer_params[q]);
   }
+  if (G.comm != nullptr && B.ev_ready == nullptr) {
+    CK(cudaEventCreateWithFlags(&B.ev_ready, cudaEventDisableTiming));
+    CK(cudaEventCreateWithFlags(&B.ev_rel, cudaEventDisableTiming));
+  }
   if (B.peers.size() != B.ranges.size()) B.peers.resize(B.ranges.size());
   if (B.peers[range_idx].empty()) ++G.n_peer_ranges;
   B.peers[range_idx] = v;
+  B.pp = true;
   return RATEL_OK;
 }
 
@@ -1660,10 +1676,13 @@ int ratel_offload_grad_chunk(int block_id, void* stream) {
         return set_error(RATEL_ESTATE, "ratel_offload_grad_chunk: block %d range %zu has no SSD file", block_id, i);
   CK(cudaEventRecord(B.ev_grad, static_cast<cudaStream_t>(stream)));
   CK(cudaStreamWaitEvent(G.s_opt, B.ev_grad, 0));
-  if (B.rs && G.comm != nullptr) {
+  if ((B.rs || B.pp) && G.comm != nullptr) {
     // Fused reduction: this rank is about to read every rank's G16 of the
-    // block.  An 8-byte allreduce after the local hand-off is the barrier --
-    // once it completes, every rank's backward has produced the block.
+    // block; fused all-gather: it is about to store its P16 slice into every
+    // rank's buffer, which a slower rank's backward may still be reading.  An
+    // 8-byte allreduce after the local hand-off is the barrier -- once it
+    // completes, every rank's backward has produced the block (and enqueued
+    // every GEMM that reads its P16 before the hand-off's event).
     CK(cudaStreamWaitEvent(G.s_comm, B.ev_grad, 0));
     NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
     CK(cudaEventRecord(B.ev_ready, G.s_comm));
@@ -1691,7 +1710,12 @@ int ratel_block_wait(int block_id, void* stream) {
   const Block& B = G.blocks[block_id];
   if (B.handed_off && !B.enqueued)
     return set_error(RATEL_ESTATE, "ratel_block_wait: block %d's update is not enqueued yet", block_id);
-  if (B.residency == RATEL_SSD && B.enqueued) RK(ssd_drain(false, B.ssd_seq));  // its ev_done is recorded
+  if (B.residency == RATEL_SSD && B.enqueued) {
+    RK(ssd_drain(false, B.ssd_seq));  // its ev_done is recorded
+    // the reader's G16 reads ran on its own streams: keep ratel_optimizer_stream()
+    // ordered after them (grad.record_stream(ratel_optimizer_stream()) contract)
+    CK(cudaStreamWaitEvent(G.s_opt, B.ev_done, 0));
+  }
   if (B.rs && G.comm != nullptr && B.enqueued) {
     // Peers read this rank's G16 too: release it only after every rank's
     // update of the block (collective: every rank calls block_wait alike).
@@ -1768,6 +1792,89 @@ int ratel_finalize(void) {
     if (s) cudaStreamSynchronize(s);
   destroy_all();
   cudaGetLastError();
+  return RATEL_OK;
+}
+
+int ratel_refresh_params(int block_id, void* stream) {
+  Nvtx nv("ratel_refresh_params %d", block_id);
+  RK(entry());
+  if (stream != nullptr) RK(check_not_capturing(stream, "ratel_refresh_params"));
+  if (G.armed || G.n_handed > 0) return set_error(RATEL_ESTATE, "ratel_refresh_params: a step is in flight");
+  if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
+    return set_error(RATEL_ESTATE, "ratel_refresh_params: block %d is not registered", block_id);
+  Block& B = G.blocks[block_id];
+  const cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  // after whatever the caller enqueued (e.g. restored states), and after every
+  // earlier update (s_opt is ordered after all of them by ratel_sync)
+  CK(cudaEventRecord(B.ev_grad, cs));
+  CK(cudaStreamWaitEvent(G.s_opt, B.ev_grad, 0));
+  const unsigned grid_max = static_cast<unsigned>(G.sms) * 4u;
+  auto launch = [&](const float* th, uint16_t* p, uint64_t n, const PeerDesc& pd) -> int {
+    const uint64_t want = std::max<uint64_t>(1, (n / 8 + kThreads - 1) / kThreads);
+    const unsigned g = static_cast<unsigned>(std::min<uint64_t>(want, grid_max));
+    refresh_p16_kernel<<<g, kThreads, 0, G.s_opt>>>(th, p, n, pd);
+    CK(cudaGetLastError());
+    ++G.launches;
+    return RATEL_OK;
+  };
+  float* stage = nullptr;  // SSD: the master is in the state file, read tile by tile
+  int rc = RATEL_OK;
+  for (size_t i = 0; i < B.ranges.size() && rc == RATEL_OK; ++i) {
+    const ratel_range& r = B.ranges[i];
+    const Slice& s = B.slices[i];
+    const uint64_t n = s.end - s.begin;
+    if (n == 0) continue;
+    uint16_t* p = static_cast<uint16_t*>(r.param_bf16) + s.begin;
+    if (B.residency != RATEL_SSD) {  // device or page-locked host master (read in place)
+      rc = launch(r.master, p, n, peer_desc(B, i, 0));
+      continue;
+    }
+    const uint64_t T = G.cfg.tile_elems;
+    if (stage == nullptr && cudaHostAlloc(&stage, T * sizeof(float), cudaHostAllocDefault) != cudaSuccess) {
+      stage = nullptr;
+      return sticky_fail(RATEL_ENOMEM, "ratel_refresh_params: staging cudaHostAlloc failed");
+    }
+    const Block::SsdRange& f = B.ssd[i];
+    if (f.fd < 0) {
+      rc = set_error(RATEL_ESTATE, "ratel_refresh_params: block %d range %zu has no SSD file", block_id, i);
+      break;
+    }
+    for (uint64_t off = 0; off < n && rc == RATEL_OK; off += T) {
+      const uint64_t len = std::min<uint64_t>(T, n - off);
+      const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
+      if (cudaStreamSynchronize(G.s_opt) != cudaSuccess) {  // the previous tile's kernel read the stage
+        rc = sticky_fail(RATEL_ECUDA, "ratel_refresh_params: %s", cudaGetErrorString(cudaGetLastError()));
+        break;
+      }
+      std::string msg;
+      rc = io_full(true, f.fd, stage, bytes, f.off + off * 4, msg);
+      if (rc != RATEL_OK) {
+        rc = sticky_fail(rc, "ratel_refresh_params: %s", msg.c_str());
+        break;
+      }
+      rc = launch(stage, p + off, len, peer_desc(B, i, off));
+    }
+  }
+  if (stage != nullptr) {
+    cudaStreamSynchronize(G.s_opt);
+    cudaFreeHost(stage);
+  }
+  if (rc != RATEL_OK) return rc;
+  CK(cudaEventRecord(B.ev_done, G.s_opt));
+  cudaEvent_t last = B.ev_done;
+  if (G.comm != nullptr) {
+    RK(allgather_block(B));  // NCCL ranges: in-place bf16 all-gather on the comm stream
+    CK(cudaStreamWaitEvent(G.s_comm, B.ev_done, 0));
+    if (B.pp)  // peer stores: every rank's refresh kernel done (collective)
+      NK(g_nccl.AllReduce(G.d_barrier, G.d_barrier, 1, ncclFloat64, ncclSum, G.comm, G.s_comm));
+    CK(cudaEventRecord(G.ev_end[3], G.s_comm));
+    last = G.ev_end[3];
+  }
+  if (stream != nullptr) {
+    CK(cudaStreamWaitEvent(cs, last, 0));
+  } else {
+    CK(cudaEventSynchronize(last));
+  }
   return RATEL_OK;
 }
 

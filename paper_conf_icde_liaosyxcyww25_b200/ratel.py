@@ -117,6 +117,7 @@ def load_library(path: str = _LIB_PATH, strict: bool = True):
         "ratel_offload_grad_chunk": (I, [I, P]),
         "ratel_sync": (I, [P]),
         "ratel_block_wait": (I, [I, P]),
+        "ratel_refresh_params": (I, [I, P]),
         "ratel_register_peer_params": (I, [I, I, ctypes.POINTER(P), I]),
         "ratel_register_peer_grads": (I, [I, I, ctypes.POINTER(P), I, D]),
         "ratel_register_ssd": (I, [I, I, I, U64]),
@@ -166,11 +167,19 @@ def _check(rc: int) -> None:
         raise RatelError(rc, (_lib.ratel_last_error() or b"").decode(errors="replace"))
 
 
+CUDA_STREAM_LEGACY = 0x1   # cudaStreamLegacy
+
+
 def _stream(s):
+    """None -> NULL (ratel_sync: block the host); a torch stream -> its
+    handle, torch's legacy default stream (handle 0) -> cudaStreamLegacy so
+    that ratel_sync(torch.cuda.current_stream()) stays stream-ordered there
+    too instead of turning into the host-blocking NULL form."""
     if s is None:
         return None
     if hasattr(s, "cuda_stream"):
-        return s.cuda_stream
+        h = s.cuda_stream
+        return h if h != 0 else CUDA_STREAM_LEGACY
     return int(s)
 
 
@@ -276,6 +285,10 @@ def ratel_block_wait(block_id: int, stream=None) -> None:
 
 def ratel_sync(stream=None) -> None:
     _check(_lib.ratel_sync(_stream(stream)))
+
+
+def ratel_refresh_params(block_id: int, stream=None) -> None:
+    _check(_lib.ratel_refresh_params(block_id, _stream(stream)))
 
 
 def ratel_finalize() -> None:
