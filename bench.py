@@ -273,8 +273,10 @@ def workload_config(args, world):
                        f"handler"}.get(args.residency, "device")
     name = {"13B": "13B", "30B": "30B", "70B": "70B (Table IV shape, 64.9B)", "175B": "175B",
             "c1": "C1 tiny block"}[shape]
+    leff = (f", L_eff = {len(sizes)} of {len(model_blocks(shape))} blocks sized to this box"
+            if getattr(args, "blocks_auto", False) else "")
     return {"workload": f"{name} GPT model states ({len(sizes)} blocks), {resid}-resident, AdamW, "
-                        f"per-block AGO hand-off" + (", clip" if args.clip > 0 else ""),
+                        f"per-block AGO hand-off" + (", clip" if args.clip > 0 else "") + leff,
             "params": P, "blocks": len(sizes), "block_params": sizes[0], "residency": resid,
             "parallelism": (f"range-sharded x{world}" + (" (fused peer-store all-gather)" if args.fused_allgather else
                                                           " (NCCL all-gather)")
@@ -1065,6 +1067,40 @@ def relaunch_or_world(args) -> int:
     return world
 
 
+def mem_available_bytes() -> int:
+    with open("/proc/meminfo") as f:
+        for line in f:
+            if line.startswith("MemAvailable:"):
+                return int(line.split()[1]) * 1024
+    raise RuntimeError("no MemAvailable in /proc/meminfo")
+
+
+def auto_blocks(args, world: int) -> int:
+    """L_eff: the most leading blocks of the shape whose
+    states fit the box.  Host residencies: the fp32 theta/m/v of ALL ranks'
+    slices (12 B/param in total) within 85 % of MemAvailable; every rank also
+    keeps the full bf16 P16 of its blocks in HBM (2 B/param), capped at 60 %
+    of a 180 GB GPU.  Device residency: (12/N + 2) B/param within 95 % of HBM."""
+    sizes = model_blocks(args.shape)
+    if args.residency == "device":
+        budget = 0.95 * 183_359 * 2 ** 20
+        per = lambda n: (12.0 / world + 2.0) * n
+    else:
+        host = 0.85 * mem_available_bytes()
+        dev = 0.60 * 183_359 * 2 ** 20
+        per = lambda n: max(12.0 * n / host, 2.0 * n / dev)
+        budget = 1.0
+    used, k = 0.0, 0
+    for n in sizes:
+        if used + per(n) > budget:
+            break
+        used += per(n)
+        k += 1
+    if k == 0:
+        raise SystemExit("--blocks auto: not even one block of this shape fits the box")
+    return k
+
+
 def share_gpu_nccl_env(rank: int) -> None:
     """--share-gpu: NCCL refuses two ranks on one device of one host ("Duplicate
     GPU"); giving each rank its own NCCL host id makes them peers on different
@@ -1085,7 +1121,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ratel", choices=["ratel", "reference"])
     ap.add_argument("--shape", default="13B", choices=list(SHAPES))
-    ap.add_argument("--blocks", type=int, default=0, help="use only the first N blocks")
+    ap.add_argument("--blocks", default="0",
+                    help="use only the first N blocks; 'auto' = L_eff, the most blocks whose states fit this box "
+                         "(host residencies: 85 %% of MemAvailable shared by all ranks; device: 95 %% of HBM)")
     ap.add_argument("--residency", default="device", choices=["device", "host", "hostcompute", "hybrid"])
     ap.add_argument("--hybrid-gpu-frac", type=float, default=0.3,
                     help="hybrid residency: fraction of each block streamed through the GPU (pinned-host tile "
@@ -1131,6 +1169,8 @@ def main():
     if args.steps < 1 or args.warmup < 0:
         raise SystemExit("need --steps >= 1")
     world = relaunch_or_world(args)
+    args.blocks_auto = args.blocks == "auto"
+    args.blocks = auto_blocks(args, world) if args.blocks_auto else int(args.blocks)
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
 

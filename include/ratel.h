@@ -149,6 +149,15 @@ typedef enum { RATEL_COMM_AUTO = 0, RATEL_COMM_NONE = 1, RATEL_COMM_NCCL = 2 } r
  *          memory: small enough to share an SM with a backward GEMM CTA while AGO overlaps them. */
 typedef enum { RATEL_UPDATE_TMA = 0, RATEL_UPDATE_LDG = 1, RATEL_UPDATE_LDG_LITE = 2 } ratel_k1_kernel;
 
+/* SSD tier I/O schedule.  DUPLEX: the reader (file -> staging) and the writer
+ * (staging -> file) threads run freely, the device's queue mixes reads and
+ * writes.  SIMPLEX: the paper's schedule for a simplex SSD link (Fig. 3b,
+ * P:L1128-1131): one transfer at a time, and the write-back of
+ * tile k starts only after the read of tile k+1 (or once no read is pending),
+ * i.e. R0 R1 W0 R2 W1 R3 W2 ... -- "Main->SSD of tensor i after SSD->Main of
+ * tensor i-1", at tile granularity. */
+typedef enum { RATEL_SSD_DUPLEX = 0, RATEL_SSD_SIMPLEX = 1 } ratel_ssd_schedule;
+
 typedef struct {
   int mode;               /* ratel_mode; default RATEL_ADAMW */
   double max_grad_norm;   /* > 0 enables the global L2-norm clip (torch clip_grad_norm_); default 0 */
@@ -170,6 +179,8 @@ typedef struct {
                              waiting for a persistent CTA; max_ctas is ignored.  Results are identical. */
   int k1_kernel;          /* ratel_k1_kernel: which update kernel (device-resident and tile updates);
                              default RATEL_UPDATE_TMA.  Results are identical. */
+  int ssd_schedule;       /* ratel_ssd_schedule: RATEL_SSD* tiers; default RATEL_SSD_DUPLEX.  Results are
+                             identical. */
 } ratel_config;
 
 /* One contiguous parameter range of a block (a flat tensor, or a block's

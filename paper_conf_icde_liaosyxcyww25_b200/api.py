@@ -82,27 +82,55 @@ class _SsdFile:
         self.fd = self.fd_buf = None
 
 
-class _SymmArena:
+class _PeerArena:
     """Data-parallel buffers for world > 1: every range's P16 and G16 carved
-    out of two flat torch symmetric-memory allocations (one rendezvous each),
-    so every rank can map every other rank's buffers -- the peer pointers the
-    fused reduce-scatter (ratel_register_peer_grads) and the fused all-gather
-    (ratel_register_peer_params) need."""
+    out of two flat allocations that every rank maps, so each rank holds the
+    peer pointers the fused reduce-scatter (ratel_register_peer_grads) and the
+    fused all-gather (ratel_register_peer_params) need.
+      peer_memory="symm": torch symmetric memory (one rendezvous per buffer;
+        one GPU per rank, NVLink peer mappings);
+      peer_memory="ipc": plain CUDA allocations exported as CUDA IPC handles
+        and opened by every rank of this node (torch's tensor-sharing
+        reduction, handles exchanged with all_gather_object) -- also works
+        when ranks share a GPU, which symmetric memory refuses."""
 
-    def __init__(self, caps, dev):
+    def __init__(self, caps, dev, peer_memory="symm"):
         import torch.distributed as dist
-        import torch.distributed._symmetric_memory as symm_mem
         self.offs, off = [], 0
         for c in caps:
             self.offs.append(off)
             off += (c + 7) // 8 * 8          # 16-byte aligned views
-        self.p16 = symm_mem.empty(max(off, 8), dtype=torch.bfloat16, device=dev)
-        self.g16 = symm_mem.empty(max(off, 8), dtype=torch.bfloat16, device=dev)
-        self.p16.zero_()
-        self.g16.zero_()
-        group = dist.group.WORLD.group_name
-        self.hp = symm_mem.rendezvous(self.p16, group)
-        self.hg = symm_mem.rendezvous(self.g16, group)
+        n = max(off, 8)
+        if peer_memory == "symm":
+            import torch.distributed._symmetric_memory as symm_mem
+            self.p16 = symm_mem.empty(n, dtype=torch.bfloat16, device=dev)
+            self.g16 = symm_mem.empty(n, dtype=torch.bfloat16, device=dev)
+            self.p16.zero_()
+            self.g16.zero_()
+            group = dist.group.WORLD.group_name
+            self.bases_p = list(symm_mem.rendezvous(self.p16, group).buffer_ptrs)
+            self.bases_g = list(symm_mem.rendezvous(self.g16, group).buffer_ptrs)
+        elif peer_memory == "ipc":
+            from torch.multiprocessing.reductions import reduce_tensor
+            self.p16 = torch.zeros(n, dtype=torch.bfloat16, device=dev)
+            self.g16 = torch.zeros(n, dtype=torch.bfloat16, device=dev)
+            torch.cuda.synchronize()
+            mine = (reduce_tensor(self.p16), reduce_tensor(self.g16))
+            allh = [None] * dist.get_world_size()
+            dist.all_gather_object(allh, mine)
+            me = dist.get_rank()
+            self.mapped = []                 # peers' tensors, kept open until this arena dies
+            self.bases_p, self.bases_g = [], []
+            for q, (hp, hg) in enumerate(allh):
+                if q == me:
+                    tp, tg = self.p16, self.g16
+                else:
+                    tp, tg = hp[0](*hp[1]), hg[0](*hg[1])
+                    self.mapped += [tp, tg]
+                self.bases_p.append(tp.data_ptr())
+                self.bases_g.append(tg.data_ptr())
+        else:
+            raise ValueError(f"peer_memory must be 'symm' or 'ipc', not {peer_memory!r}")
         self.next = 0
 
     def take(self, cap):
@@ -110,7 +138,7 @@ class _SymmArena:
         self.next += 1
         o = self.offs[k]
         return (self.p16[o:o + cap], self.g16[o:o + cap],
-                [b + 2 * o for b in self.hp.buffer_ptrs], [b + 2 * o for b in self.hg.buffer_ptrs])
+                [b + 2 * o for b in self.bases_p], [b + 2 * o for b in self.bases_g])
 
 
 class _Range:
@@ -225,14 +253,15 @@ class Ratel_Optimizer:
     library, so each rank's update kernel reduces the N local gradients of its
     slice (mean, fp64, R17) and stores its P16 slice into every
     rank's copy (fused reduce-scatter + all-gather over NVLink; residency
-    "device" or "host").  data_parallel="reduced" is for callers whose
+    "device" or "host"; peer_memory="ipc" maps plain allocations through CUDA
+    IPC instead, e.g. when ranks share a GPU).  data_parallel="reduced" is for callers whose
     gradients are already identical on every rank when the hook fires (the
     library then only all-gathers P16 over NCCL, R11).  Both sides of a step
     are collective: every rank hands off the same units in the same order."""
 
     def __init__(self, blocks, lr=1e-3, betas=(0.9, 0.999), eps=1e-8, weight_decay=1e-2,
                  residency="device", no_decay=None, first_block_id=0, granularity="block", ssd_path=None,
-                 hybrid_gpu_frac=0.3, data_parallel="fused"):
+                 hybrid_gpu_frac=0.3, data_parallel="fused", peer_memory="symm"):
         import torch.distributed as dist
         distributed = dist.is_available() and dist.is_initialized()
         world = dist.get_world_size() if distributed else 1
@@ -269,7 +298,7 @@ class Ratel_Optimizer:
         arena = None
         if fused_dp:
             caps = [R.ratel_padded_numel(sum(p.numel() for p in ps), world) for groups in units for ps, _ in groups]
-            arena = _SymmArena(caps, dev)
+            arena = _PeerArena(caps, dev, peer_memory)
         ssd = residency in ("ssd", "ssd_hostcompute")
         if ssd and not ssd_path:
             raise ValueError(f'residency="{residency}" needs ssd_path (the state file to create)')

@@ -114,6 +114,7 @@ struct SsdJob {
   std::vector<cudaEvent_t> wait;  // host-waited before the block's states are read
 };
 struct SsdTile {
+  uint64_t seq = 0;  // ring order (E.ring_k at its read)
   int slot = 0, fd = -1;
   uint64_t foff = 0, stride = 0, bytes = 0;
   bool host = false;  // updated by the CPU handler in the staging slot (no D2H to wait for)
@@ -127,6 +128,12 @@ struct SsdEngine {
   int slot_busy[kMaxDepth] = {};  // a tile in this slot still awaits its write-back
   bool stop = false;
   bool reader_done = false;  // the writer drains until the reader can queue no more tiles
+  // RATEL_SSD_SIMPLEX: one file transfer at a time (disk_busy), and tile k's
+  // write-back waits for tile k+1's read (tiles_read > k+1) unless no read is
+  // pending (reader idle with an empty job queue).
+  bool disk_busy = false;
+  bool reader_idle = true;
+  uint64_t tiles_read = 0;   // tiles whose three arrays have been read (ring order)
   uint64_t jobs_in = 0, jobs_out = 0, tiles_in = 0, tiles_out = 0;
   int err = 0;
   std::string msg;
@@ -685,6 +692,24 @@ double now_s() {
   return ts.tv_sec + 1e-9 * ts.tv_nsec;
 }
 
+bool ssd_simplex() { return G.cfg.ssd_schedule == RATEL_SSD_SIMPLEX; }
+
+// Simplex schedule: take / release the one-transfer-at-a-time disk token.
+void disk_acquire(SsdEngine& E) {
+  if (!ssd_simplex()) return;
+  std::unique_lock<std::mutex> lk(E.mu);
+  E.cv.wait(lk, [&] { return !E.disk_busy; });
+  E.disk_busy = true;
+}
+void disk_release(SsdEngine& E, bool read_done) {
+  {
+    std::lock_guard<std::mutex> lk(E.mu);
+    if (ssd_simplex()) E.disk_busy = false;
+    if (read_done) ++E.tiles_read;
+  }
+  E.cv.notify_all();
+}
+
 int io_full(bool rd, int fd, void* buf, uint64_t bytes, uint64_t off, std::string& msg) {
   uint8_t* p = static_cast<uint8_t*>(buf);
   while (bytes > 0) {
@@ -750,12 +775,17 @@ int ssd_run_job_cpu(SsdEngine& E, Block& B, std::string& msg) {
       }
       float* h = E.h_ring + 3ull * slot * T;
       const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
+      disk_acquire(E);
       const double t0 = now_s();
       for (int a = 0; a < 3; ++a) {
         const int rc = io_full(true, f.fd, h + a * T, bytes, f.off + a * f.stride + off * 4, msg);
-        if (rc != RATEL_OK) return rc;
+        if (rc != RATEL_OK) {
+          disk_release(E, false);
+          return rc;
+        }
       }
       E.read_s += now_s() - t0;
+      disk_release(E, true);
       E.read_bytes += 3 * bytes;
       HostAdamArgs a{};
       a.g = B.h_g[i] + off;
@@ -779,6 +809,7 @@ int ssd_run_job_cpu(SsdEngine& E, Block& B, std::string& msg) {
         std::lock_guard<std::mutex> lk(E.mu);
         E.slot_busy[slot] = 1;
         SsdTile t;
+        t.seq = E.ring_k;
         t.slot = slot;
         t.fd = f.fd;
         t.foff = f.off + off * 4;
@@ -826,12 +857,17 @@ int ssd_run_job(SsdEngine& E, const SsdJob& job, std::string& msg) {
       float* h = E.h_ring + 3ull * slot * T;
       float* d = E.d_ring + 3ull * slot * T;
       const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
+      disk_acquire(E);
       const double t0 = now_s();
       for (int a = 0; a < 3; ++a) {
         const int rc = io_full(true, f.fd, h + a * T, bytes, f.off + a * f.stride + off * 4, msg);
-        if (rc != RATEL_OK) return rc;
+        if (rc != RATEL_OK) {
+          disk_release(E, false);
+          return rc;
+        }
       }
       E.read_s += now_s() - t0;
+      disk_release(E, true);
       E.read_bytes += 3 * bytes;
       for (int a = 0; a < 3; ++a) SK(cudaMemcpyAsync(d + a * T, h + a * T, len * 4, cudaMemcpyHostToDevice, E.s_in));
       SK(cudaEventRecord(E.ev_h2d[slot], E.s_in));
@@ -861,6 +897,7 @@ int ssd_run_job(SsdEngine& E, const SsdJob& job, std::string& msg) {
         std::lock_guard<std::mutex> lk(E.mu);
         E.slot_busy[slot] = 1;
         SsdTile t;
+        t.seq = E.ring_k;
         t.slot = slot;
         t.fd = f.fd;
         t.foff = f.off + off * 4;
@@ -894,6 +931,8 @@ void ssd_reader_main(SsdEngine* E) {
     SsdJob job;
     {
       std::unique_lock<std::mutex> lk(E->mu);
+      E->reader_idle = true;
+      E->cv.notify_all();  // a simplex write-back may be waiting for "no read pending"
       E->cv.wait(lk, [&] { return E->stop || !E->jobs.empty(); });
       if (E->jobs.empty()) {  // stop
         E->reader_done = true;
@@ -903,6 +942,7 @@ void ssd_reader_main(SsdEngine* E) {
       }
       job = E->jobs.front();
       E->jobs.pop_front();
+      E->reader_idle = false;
     }
     bool failed;
     {
@@ -938,6 +978,17 @@ void ssd_writer_main(SsdEngine* E) {
       E->wq.pop_front();
       failed = E->err != 0;
     }
+    if (!failed && ssd_simplex()) {
+      // the paper's simplex order: write tile k back only after tile k+1 was
+      // read (or no read is pending), and never during another transfer
+      std::unique_lock<std::mutex> lk(E->mu);
+      E->cv.wait(lk, [&] {
+        const bool next_read = E->tiles_read > t.seq + 1 ||
+                               (E->reader_idle && E->jobs.empty()) || E->err != 0;
+        return next_read && !E->disk_busy;
+      });
+      E->disk_busy = true;
+    }
     if (!failed) {
       std::string m;
       int rc = RATEL_OK;
@@ -952,6 +1003,7 @@ void ssd_writer_main(SsdEngine* E) {
         rc = io_full(false, t.fd, const_cast<float*>(h + a * T), t.bytes, t.foff + a * t.stride, m);
       E->write_s += now_s() - t0;
       E->write_bytes += 3 * t.bytes;
+      if (ssd_simplex()) disk_release(*E, false);
       if (rc != RATEL_OK) ssd_fail(*E, rc, "SSD writer: " + m);
     }
     {
@@ -1174,6 +1226,8 @@ int validate_config(const ratel_config& c) {
   if (c.cta_tiles < 0) return set_error(RATEL_EINVAL, "cfg.cta_tiles must be >= 0");
   if (c.k1_kernel != RATEL_UPDATE_TMA && c.k1_kernel != RATEL_UPDATE_LDG && c.k1_kernel != RATEL_UPDATE_LDG_LITE)
     return set_error(RATEL_EINVAL, "cfg.k1_kernel");
+  if (c.ssd_schedule != RATEL_SSD_DUPLEX && c.ssd_schedule != RATEL_SSD_SIMPLEX)
+    return set_error(RATEL_EINVAL, "cfg.ssd_schedule");
   return RATEL_OK;
 }
 
@@ -1330,6 +1384,7 @@ void ratel_default_config(ratel_config* cfg) {
   cfg->update_streams = 2;
   cfg->cta_tiles = 0;
   cfg->k1_kernel = RATEL_UPDATE_TMA;
+  cfg->ssd_schedule = RATEL_SSD_DUPLEX;
 }
 
 uint64_t ratel_padded_numel(uint64_t numel, int world_size) {

@@ -41,6 +41,8 @@ RATEL_COMM_NCCL = 2
 RATEL_UPDATE_TMA = 0
 RATEL_UPDATE_LDG = 1
 RATEL_UPDATE_LDG_LITE = 2
+RATEL_SSD_DUPLEX = 0
+RATEL_SSD_SIMPLEX = 1
 RATEL_MAX_BLOCKS = 4096
 RATEL_MAX_RANGES_PER_BLOCK = 32
 
@@ -69,6 +71,7 @@ class ratel_config(ctypes.Structure):
         ("update_streams", ctypes.c_int),
         ("cta_tiles", ctypes.c_int),
         ("k1_kernel", ctypes.c_int),
+        ("ssd_schedule", ctypes.c_int),
     ]
 
 

@@ -1,0 +1,168 @@
+"""The paper's user API under data parallelism on a REAL NCCL communicator.
+
+Two ranks (one GPU each, or -- on a one-GPU box -- both on cuda:0 with
+distinct NCCL host ids, see tests/test_nccl_ranks_gpu.py) run
+Ratel_init / Ratel_Optimizer(data_parallel="fused") / Ratel_hook on the same
+model with DIFFERENT micro-batches.  P16 and G16 live in memory every rank
+maps (torch symmetric memory, or CUDA IPC when the ranks share a GPU); each
+post-accumulate hook hands the rank's LOCAL gradient off, the
+library's NCCL barrier orders the ranks, and every rank's update kernel
+reduces the two local gradients of its slice (mean, R17) and stores
+its P16 slice into both ranks' buffers.  Checked: the concatenated slices
+against the oracle's data-parallel step (oracle.adam_step_dp on the ranks'
+recorded local gradients) under R13, identical P16 on both ranks, and
+state_dict / load_state_dict (ratel_refresh_params) resuming bitwise.
+"""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from tests.tolerance import check_range
+
+pytestmark = pytest.mark.gpu
+
+D, NB, STEPS = 64, 2, 3
+HPK = dict(lr=2e-3, beta1=0.9, beta2=0.99, eps=1e-8, weight_decay=0.05)
+
+
+def _free_port():
+    with socket.socket() as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+class Block(torch.nn.Module):
+    def __init__(self, d):
+        super().__init__()
+        self.fc1 = torch.nn.Linear(d, 4 * d)
+        self.fc2 = torch.nn.Linear(4 * d, d)
+        self.ln = torch.nn.LayerNorm(d)
+
+    def forward(self, x):
+        return x + self.fc2(torch.nn.functional.gelu(self.fc1(self.ln(x))))
+
+
+def _flat_ranges(model):
+    """Initial fp32 values of every range, in Ratel_Optimizer's order
+    (per block: decayed params, then the no-decay ones)."""
+    out = []
+    for b in model:
+        ps = list(b.parameters())
+        for group in ([p for p in ps if p.ndim > 1], [p for p in ps if p.ndim <= 1]):
+            out.append(torch.cat([p.detach().reshape(-1).float().cpu() for p in group]).numpy())
+    return out
+
+
+def _rank_main(rank, world, shared, port, res_q, peer_memory):
+    if shared:
+        os.environ["NCCL_HOSTID"] = f"ratel-api-rank{rank}"
+        os.environ["NCCL_SOCKET_IFNAME"] = "lo"
+        os.environ["NCCL_IB_DISABLE"] = "1"
+    import torch.distributed as dist
+
+    from paper_conf_icde_liaosyxcyww25_b200.api import Ratel_hook, Ratel_init, Ratel_Optimizer
+
+    dev_i = 0 if shared else rank
+    torch.cuda.set_device(dev_i)
+    dev = torch.device("cuda", dev_i)
+    dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world,
+                            device_id=dev)
+    try:
+        torch.manual_seed(0)                               # the same model on every rank
+        model = torch.nn.Sequential(*[Block(D) for _ in range(NB)]).to(dev)
+        init = _flat_ranges(model)
+        gen = torch.Generator(device=dev)
+        gen.manual_seed(100 + rank)                        # a different micro-batch per rank
+        xs = [torch.randn(32, D, device=dev, dtype=torch.bfloat16, generator=gen) for _ in range(STEPS + 2)]
+        with Ratel_init():
+            opt = Ratel_Optimizer([list(b.parameters()) for b in model], lr=HPK["lr"],
+                                  betas=(HPK["beta1"], HPK["beta2"]), eps=HPK["eps"],
+                                  weight_decay=HPK["weight_decay"], data_parallel="fused",
+                                  peer_memory=peer_memory)
+            Ratel_hook(opt)
+            ranges = [r for rs in opt.blocks for r in rs]
+            local_grads = []
+            for t in range(STEPS):
+                opt.begin_step()
+                model(xs[t]).float().pow(2).mean().backward()
+                torch.cuda.synchronize()
+                local_grads.append([r.g16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16)
+                                    for r in ranges])
+                opt.end_step()
+                torch.cuda.synchronize()
+            out = []
+            for r in ranges:
+                beg, end = r.slice
+                out.append(dict(p32=r.master[:end - beg].cpu().numpy(), m32=r.m[:end - beg].cpu().numpy(),
+                                v32=r.v[:end - beg].cpu().numpy(),
+                                p16=r.p16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16)))
+            # resume: save, scramble P16 and states, load -> P16 rebuilt and gathered, then one more step
+            sd = opt.state_dict()
+            for r in ranges:
+                r.p16.fill_(3.0)
+                r.master.fill_(9.0)
+            torch.cuda.synchronize()
+            dist.barrier()
+            opt.load_state_dict(sd)
+            torch.cuda.synchronize()
+            reloaded = [r.p16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16) for r in ranges]
+            opt.remove_hooks()
+            del opt
+        res_q.put((rank, init, local_grads, out, reloaded))
+    except BaseException as e:
+        res_q.put((rank, repr(e), None, None, None))
+        raise
+    finally:
+        try:
+            dist.barrier()
+            dist.destroy_process_group()
+        except Exception:
+            pass
+
+
+@pytest.mark.parametrize("peer_memory", ["ipc", "symm"])
+def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
+    """peer_memory="symm" (torch symmetric memory) needs a GPU per rank; on a
+    one-GPU box only the CUDA-IPC mapping runs."""
+    n = torch.cuda.device_count()
+    world, shared = (2, n < 2)
+    if shared and peer_memory == "symm":
+        pytest.skip("torch symmetric memory refuses ranks that share a GPU")
+    ctx = torch.multiprocessing.get_context("spawn")
+    res_q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, res_q, peer_memory)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    try:
+        for _ in range(world):
+            r, init, grads, out, reloaded = res_q.get(timeout=600)
+            assert not isinstance(init, str), f"rank {r}: {init}"
+            res[r] = (init, grads, out, reloaded)
+    finally:
+        for p in procs:
+            p.join(timeout=120)
+            if p.is_alive():
+                p.kill()
+    assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
+    init = res[0][0]
+    for k in range(len(init)):
+        assert np.array_equal(res[1][0][k], init[k])          # same model on both ranks
+    wd = [1, 0] * NB                                           # weights decay, biases / LN do not
+    refs = [oracle.Range.fresh(a.astype(np.float32), wd[k]) for k, a in enumerate(init)]
+    for t in range(STEPS):
+        assert not all(np.array_equal(res[0][1][t][k], res[1][1][t][k]) for k in range(len(refs)))
+        oracle.adam_step_dp(refs, [[res[q][1][t][k] for q in range(world)] for k in range(len(refs))],
+                            1.0 / world, oracle.hparams(step=t + 1, **HPK))
+    for k, ref in enumerate(refs):
+        got = {f: np.concatenate([res[q][2][k][f] for q in range(world)]) for f in ("p32", "m32", "v32")}
+        got["p16"] = res[0][2][k]["p16"]
+        check_range(got, ref, own_rne=oracle.bf16_rne, what=f"api dp range {k}")
+        assert np.array_equal(res[1][2][k]["p16"], res[0][2][k]["p16"])
+        for q in range(world):                                 # resume: P16 rebuilt from the masters
+            assert np.array_equal(res[q][3][k], oracle.bf16_rne(got["p32"])), (k, q)

@@ -190,3 +190,23 @@ def test_ssd_host_compute_nonfinite_norm_reported(cuda_dev, tmp_path):
         assert e.value.code == R.RATEL_ENONFINITE
     assert np.isnan(b.gpu_state(0)["p32"]).all()
     b.close()
+
+
+@pytest.mark.parametrize("cpu", [False, True])
+def test_ssd_simplex_schedule_bitwise(cuda_dev, tmp_path, cpu):
+    """cfg.ssd_schedule = RATEL_SSD_SIMPLEX (the paper's simplex order, Fig. 3b
+    P:L1128-1131: one transfer at a time, write-back of tile k after the read of
+    tile k+1) changes only when the file is touched: bitwise the device /
+    HOST_COMPUTE result, with clipping and one state file for all blocks."""
+    base, ssd = 0, []
+    for i, n in enumerate(SIZES):
+        b = SsdBlock(i, [n], cuda_dev, tmp_path / "states.bin", base=base, cpu=cpu)
+        base = b.file_bytes
+        ssd.append(b)
+    run(ssd, 3, max_norm=1e-3, tile_elems=TILE, pipeline_depth=2, ssd_schedule=R.RATEL_SSD_SIMPLEX,
+        host_threads=4)
+    ref = [GpuBlock(i, [n], cuda_dev, host_compute=cpu) for i, n in enumerate(SIZES)]
+    run(ref, 3, max_norm=1e-3, host_threads=4)
+    assert_bitwise(snapshot(ssd), snapshot(ref))
+    for b in ssd:
+        b.close()
