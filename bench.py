@@ -851,7 +851,8 @@ def run_e2e_device(args, R, torch, dev, model, sizes, order, t, world):
     ms = max_over_ranks(torch, e0.elapsed_time(e1), world, dev)
     own = sum(e - b for (b, e) in model.slices)
     P = sum(sizes)
-    link = host_link_probe(torch, dev)
+    host_link_probe(torch, dev)
+    link = best_link()
     moved = 4 * own   # 2 B/param in, 2 B/param out, this rank
     achieved = moved / (ms / K / 1e3) / 1e9
     return {"value": P * K / (ms / 1e3), "unit": UNIT, "h2d_bytes_per_step": int(2 * own * world),
@@ -893,12 +894,14 @@ def offdevice_roofline(args, torch, dev, own_params_per_s, k1_roof):
     k1 = {k: v for k, v in k1_roof.items() if k not in ("traffic", "ncu_dram_pct_of_peak")}
     legs = {}
     if f > 0:
-        link = host_link_probe(torch, dev)
+        host_link_probe(torch, dev)
+        link = best_link()
         bpp = 24 * f + 4 * (1 - f)
         a = bpp * own_params_per_s / 1e9
         legs["host_link"] = {"achieved": a, "peak": link["duplex"], "frac": a / link["duplex"],
                              "algorithmic_bytes_per_param": bpp, "probe": link,
-                             "peak_source": "this run's pinned H2D || D2H probe on two streams"}
+                             "peak_source": "best of this run's pinned H2D || D2H probes on two streams "
+                                            "(start-up and after the measurement)", "probes": list(LINK_PROBES)}
     if f < 1:
         probe = host_dram_probe()
         bpp = 24 * f + 32 * (1 - f)
@@ -917,7 +920,17 @@ def offdevice_roofline(args, torch, dev, own_params_per_s, k1_roof):
             "peak_source": b["peak_source"], **legs, "k1": k1}
 
 
-def host_link_probe(torch, dev, nbytes=1 << 30, reps=3):
+LINK_PROBES = []   # every host_link_probe of this run (the roofline peak is their best)
+
+
+def best_link():
+    """Element-wise best of every host-link probe taken in this run (one at
+    start-up, one beside each measurement): the duplex probe of a single run
+    varied 79-100 GB/s on one box, so the peak is the best observed."""
+    return {k: max(p[k] for p in LINK_PROBES) for k in ("h2d", "d2h", "duplex")}
+
+
+def host_link_probe(torch, dev, nbytes=1 << 30, reps=5):
     """Measured duplex host-link bandwidth on this box (pinned H2D and D2H
     concurrently on two streams): the e2e roofline denominator."""
     n = nbytes // 4
@@ -949,6 +962,7 @@ def host_link_probe(torch, dev, nbytes=1 << 30, reps=3):
         moved = nbytes * (2 if name == "duplex" else 1)
         best[name] = moved / (min(ts) / 1e3) / 1e9
     del h1, h2, d1, d2
+    LINK_PROBES.append(dict(best))
     return best
 
 
@@ -1016,7 +1030,8 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
         h2d = (12 * own + 2 * own) * world            # states in + grads in (all ranks)
         d2h = (12 * own + 2 * own) * world            # states out + this rank's P16 slice (all ranks)
         val = P * K / (ms / 1e3)
-        link = host_link_probe(torch, dev)
+        host_link_probe(torch, dev)
+        link = best_link()
         achieved = (h2d + d2h) / world / (ms / K / 1e3) / 1e9
         res = {"value": val, "unit": UNIT, "h2d_bytes_per_step": int(h2d), "d2h_bytes_per_step": int(d2h),
                "ms_per_step": ms / K, "steps": K, "params": P, "blocks": n_blk,
@@ -1213,6 +1228,8 @@ def main():
     cfg.staging = {"pipelined": R.RATEL_STAGING_PIPELINED, "serialized": R.RATEL_STAGING_SERIALIZED,
                    "zero_copy": R.RATEL_STAGING_ZERO_COPY}[args.staging]
     cfg.k1_kernel = args.k1_kernel
+    if not args.no_e2e or args.residency != "device":
+        host_link_probe(torch, dev)          # start-up probe, before 100+ GB of states are pinned
     init_lib(R, torch, local, rank, world, cfg)
     sampler = ClockSampler(gpu_uuid(torch, dev)) if rank == 0 else None
     try:

@@ -213,10 +213,13 @@ typedef struct {
 void ratel_default_config(ratel_config* cfg);
 
 /* Writes a 128-byte NCCL unique id (rank 0 calls it and broadcasts the bytes
- * through the caller's process group).  RATEL_ENCCL if NCCL cannot be loaded. */
+ * through the caller's process group).  RATEL_ENCCL if NCCL cannot be loaded.
+ * (Multi-GPU bootstrap: the paper's multi-GPU setting, §V-G, uses
+ * no particular mechanism; NCCL over NVLink per BASELINE.json's north star.) */
 int ratel_get_nccl_unique_id(void* out128);
 
-/* Creates the optimizer/copy/comm streams (the optimizer stream at the
+/* Fig. 4's `Ratel_init()` (§IV-E): creates the
+ * optimizer/copy/comm streams (the optimizer stream at the
  * lowest priority), events and, for world_size > 1, the NCCL communicator.
  * device: CUDA ordinal this process drives.  nccl_unique_id: 128 bytes, NULL
  * when world_size == 1 (or cfg->comm == RATEL_COMM_NONE).  cfg: NULL = defaults.  RATEL_ESTATE if already
@@ -224,7 +227,10 @@ int ratel_get_nccl_unique_id(void* out128);
 int ratel_init(int device, int rank, int world_size, const void* nccl_unique_id,
                const ratel_config* cfg);
 
-/* Registers block `block_id` (0 <= id < RATEL_MAX_BLOCKS, each id once) made
+/* Fig. 4's `Ratel_Optimizer(...)` wrapping: registers the model
+ * states of one handler unit -- the paper's "tensor i" / transformer block
+ * (P:L1038-1041), P32 + OS32 + G16 + P16 of Table II.
+ * Registers block `block_id` (0 <= id < RATEL_MAX_BLOCKS, each id once) made
  * of n_ranges (1..RATEL_MAX_RANGES_PER_BLOCK) ranges, all with the given
  * residency (ratel_residency).  Validates pointer kinds (device pointers on
  * this device; pinned host for RATEL_PINNED_HOST / RATEL_HOST_COMPUTE --
@@ -292,14 +298,17 @@ int ratel_register_ssd(int block_id, int range_idx, int fd, uint64_t offset);
  * arrays of the rank's slice; 0 for an empty slice).  Pure host function. */
 uint64_t ratel_ssd_range_bytes(uint64_t numel, int world_size, int rank);
 
-/* Arms optimizer step `step` (1-based t, strictly increasing across steps)
+/* The optimizer of the iteration (Adam [44]; §II):
+ * arms optimizer step `step` (1-based t, strictly increasing across steps)
  * with the given hyperparameters (0 <= beta < 1, lr, eps, wd >= 0, finite).
  * Blocks already handed off in this step are enqueued now (deferred mode);
  * blocks handed off later are enqueued at their hand-off (AGO). */
 int ratel_adam_step(double lr, double beta1, double beta2, double eps, double weight_decay,
                     int64_t step);
 
-/* "Active message" for block `block_id`: its gradient is complete on
+/* Active gradient offloading's "active message" (§IV-C: the
+ * handler of tensor i runs "upon ... receiving the offloaded gradients",
+ * which arrive "with a decreasing index") for block `block_id`: its gradient is complete on
  * `stream` (a cudaStream_t, NULL = legacy default stream).  Records an event
  * on `stream`; the optimizer stream waits on it -- no host blocking, no data
  * movement.  RATEL_ESTATE if the block was already handed off this step or
@@ -328,14 +337,17 @@ int ratel_block_wait(int block_id, void* stream);
  * blocking sync returns RATEL_ENONFINITE if the global norm was not finite. */
 int ratel_sync(void* stream);
 
-/* Waits for outstanding work, destroys everything the library created and
+/* End of training (the exit of Fig. 4's `with Ratel_init():`):
+ * waits for outstanding work, destroys everything the library created and
  * clears all registrations and the sticky error. */
 int ratel_finalize(void);
 
 /* Message describing the last error on this thread ("" if none). */
 const char* ratel_last_error(void);
 
-/* Capacity of a range's param buffer for world_size ranks: numel rounded up
+/* Range partition of the multi-GPU path (north star: "each GPU owning a
+ * contiguous shard of optimizer state", R12).
+ * Capacity of a range's param buffer for world_size ranks: numel rounded up
  * to a multiple of 8*world_size (each rank's slice is a multiple of 8
  * elements, keeping 16-byte alignment).  Pure host function. */
 uint64_t ratel_padded_numel(uint64_t numel, int world_size);
@@ -364,10 +376,13 @@ int ratel_refresh_params(int block_id, void* stream);
 void* ratel_optimizer_stream(void);
 
 /* Blocking: the global sum of squared gradients of the last clip-mode step
- * (after the allreduce).  RATEL_ESTATE if clipping is off. */
+ * (after the allreduce; clipping per DESIGN.md R9 -- the paper is silent,
+ * the north star asks for "optional grad-norm clipping").  RATEL_ESTATE if
+ * clipping is off. */
 int ratel_get_grad_sumsq(double* out);
 
-/* Page-locked host memory for RATEL_PINNED_HOST / RATEL_HOST_COMPUTE states:
+/* Page-locked host memory for RATEL_PINNED_HOST / RATEL_HOST_COMPUTE states
+ * (the paper keeps P32/OS32 off the GPU, §III-A):
  * exactly `bytes` (cudaHostAlloc, portable), 64-byte aligned; *out = NULL on
  * failure (RATEL_ENOMEM, not sticky).  Frameworks' pinned allocators may round
  * large blocks up (torch: powers of two), which does not fit 100+ GB of

@@ -299,6 +299,7 @@ class Ratel_Optimizer:
         if fused_dp:
             caps = [R.ratel_padded_numel(sum(p.numel() for p in ps), world) for groups in units for ps, _ in groups]
             arena = _PeerArena(caps, dev, peer_memory)
+        self._arena = arena                  # keeps the peer mappings open for the optimizer's lifetime
         ssd = residency in ("ssd", "ssd_hostcompute")
         if ssd and not ssd_path:
             raise ValueError(f'residency="{residency}" needs ssd_path (the state file to create)')

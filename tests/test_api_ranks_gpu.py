@@ -64,7 +64,15 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
         os.environ["NCCL_IB_DISABLE"] = "1"
     import torch.distributed as dist
 
+    from paper_conf_icde_liaosyxcyww25_b200 import ratel as RR
     from paper_conf_icde_liaosyxcyww25_b200.api import Ratel_hook, Ratel_init, Ratel_Optimizer
+    handoffs = []
+    orig = RR.ratel_offload_grad_chunk
+
+    def traced(bid, stream=None):                      # record the hand-off order (a collective order)
+        handoffs.append((bid, getattr(stream, "cuda_stream", stream)))
+        return orig(bid, stream)
+    RR.ratel_offload_grad_chunk = traced
 
     dev_i = 0 if shared else rank
     torch.cuda.set_device(dev_i)
@@ -92,6 +100,17 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
                 torch.cuda.synchronize()
                 local_grads.append([r.g16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16)
                                     for r in ranges])
+                if t == 0:   # what this rank sees through its mapping of the peer's G16
+                    dist.barrier()
+                    q = 1 - rank
+                    peer_view = []
+                    for r in ranges:
+                        ptr = r.peer_g16[q]
+                        owner = [m for m in opt_arena(opt).mapped + [opt_arena(opt).g16]
+                                 if m.data_ptr() <= ptr < m.data_ptr() + 2 * m.numel()]
+                        base = owner[0]
+                        off = (ptr - base.data_ptr()) // 2
+                        peer_view.append(base[off:off + r.numel].view(torch.int16).cpu().numpy().view(np.uint16))
                 opt.end_step()
                 torch.cuda.synchronize()
             out = []
@@ -112,9 +131,9 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
             reloaded = [r.p16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16) for r in ranges]
             opt.remove_hooks()
             del opt
-        res_q.put((rank, init, local_grads, out, reloaded))
+        res_q.put((rank, init, local_grads, out, reloaded, peer_view, handoffs))
     except BaseException as e:
-        res_q.put((rank, repr(e), None, None, None))
+        res_q.put((rank, repr(e), None, None, None, None, None))
         raise
     finally:
         try:
@@ -122,6 +141,31 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
             dist.destroy_process_group()
         except Exception:
             pass
+
+
+def opt_arena(opt):
+    return opt._arena
+
+
+def _diagnose(init, res, world, k, got):
+    """Which gradient did the library use for range k?  Fraction of theta
+    elements within R13 of the oracle fed with each candidate."""
+    wd = [1, 0] * NB
+    n = init[k].size
+    cands = {"mean": lambda t: [[res[q][1][t][k] for q in range(world)]],
+             "sum": lambda t: [[res[q][1][t][k] for q in range(world)]],
+             "rank0_local": lambda t: [[res[0][1][t][k]]],
+             "rank1_local": lambda t: [[res[1][1][t][k]]],
+             "zero": lambda t: [[np.zeros(n, np.uint16)]]}
+    out = {}
+    for name, gq in cands.items():
+        ref = oracle.Range.fresh(init[k].astype(np.float32), wd[k])
+        for t in range(STEPS):
+            scale = 1.0 if name != "mean" else 1.0 / world
+            oracle.adam_step_dp([ref], gq(t), scale, oracle.hparams(step=t + 1, **HPK))
+        ok = np.abs(got["p32"].astype(np.float64) - ref.p32) <= 1e-5 * ref.theta_bar
+        out[name] = round(float(ok.mean()), 4)
+    return out
 
 
 @pytest.mark.parametrize("peer_memory", ["ipc", "symm"])
@@ -141,9 +185,9 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
     res = {}
     try:
         for _ in range(world):
-            r, init, grads, out, reloaded = res_q.get(timeout=600)
+            r, init, grads, out, reloaded, peer_view, handoffs = res_q.get(timeout=600)
             assert not isinstance(init, str), f"rank {r}: {init}"
-            res[r] = (init, grads, out, reloaded)
+            res[r] = (init, grads, out, reloaded, peer_view, handoffs)
     finally:
         for p in procs:
             p.join(timeout=120)
@@ -151,6 +195,11 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
                 p.kill()
     assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
     init = res[0][0]
+    # the hand-off order (each hand-off is a barrier on the library's communicator) is the same on both ranks
+    assert [h[0] for h in res[0][5]] == [h[0] for h in res[1][5]], (res[0][5], res[1][5])
+    for q in range(world):   # the mapping of the peer's G16 shows the peer's gradient
+        for k in range(len(init)):
+            assert np.array_equal(res[q][4][k], res[1 - q][1][0][k]), ("peer view", q, k)
     for k in range(len(init)):
         assert np.array_equal(res[1][0][k], init[k])          # same model on both ranks
     wd = [1, 0] * NB                                           # weights decay, biases / LN do not
@@ -162,7 +211,10 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
     for k, ref in enumerate(refs):
         got = {f: np.concatenate([res[q][2][k][f] for q in range(world)]) for f in ("p32", "m32", "v32")}
         got["p16"] = res[0][2][k]["p16"]
-        check_range(got, ref, own_rne=oracle.bf16_rne, what=f"api dp range {k}")
+        try:
+            check_range(got, ref, own_rne=oracle.bf16_rne, what=f"api dp range {k}")
+        except AssertionError as e:
+            raise AssertionError(f"{e}; closest hypothesis: {_diagnose(init, res, world, k, got)}") from None
         assert np.array_equal(res[1][2][k]["p16"], res[0][2][k]["p16"])
         for q in range(world):                                 # resume: P16 rebuilt from the masters
             assert np.array_equal(res[q][3][k], oracle.bf16_rne(got["p32"])), (k, q)

@@ -37,6 +37,8 @@ from tests.tolerance import check_range
 pytestmark = pytest.mark.gpu
 
 SIZES = [300_001, 65_560, 1_000_003, 24]
+BLOCKS = [[n] for n in SIZES]                         # one range per block
+BLOCKS_MULTI = [[300_001, 24, 4_104], [65_560, 1_000_003]]   # several ranges per block (weights + biases)
 STEPS = 3
 HPK = dict(lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, weight_decay=1e-2)
 
@@ -56,7 +58,12 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q):
+def _split(g, sizes):
+    offs = np.concatenate([[0], np.cumsum(sizes)]).astype(int)
+    return [g[offs[j]:offs[j + 1]] for j in range(len(sizes))]
+
+
+def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q, blocks_spec=BLOCKS):
     if shared:   # distinct NCCL "hosts" on one GPU, loopback sockets (set before any communicator)
         os.environ["NCCL_HOSTID"] = f"ratel-test-rank{rank}"
         os.environ["NCCL_SOCKET_IFNAME"] = "lo"
@@ -78,10 +85,10 @@ def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q):
     try:
         got_rank, got_world = rdist.init_distributed(dev_i, cfg)
         assert (got_rank, got_world) == (rank, world)
-        blocks = [GpuBlock(i, [n], dev, pinned=pinned, world=world, rank=rank) for i, n in enumerate(SIZES)]
+        blocks = [GpuBlock(i, sz, dev, pinned=pinned, world=world, rank=rank) for i, sz in enumerate(blocks_spec)]
         fused = mode == "fused"
         if fused:                                   # every rank's G16 / P16 mapped here (CUDA IPC)
-            mine = [(b.g16[0], b.p16[0]) for b in blocks]
+            mine = [[(b.g16[j], b.p16[j]) for j in range(len(b.sizes))] for b in blocks]
             for q in range(world):
                 if q != rank:
                     chans[(rank, q)].put(mine)
@@ -93,17 +100,18 @@ def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q):
         for b in blocks:
             b.register()
             if fused:
-                R.ratel_register_peer_grads(b.id, 0, [peers[q][b.id][0].data_ptr() for q in range(world)],
-                                            1.0 / world)
-                R.ratel_register_peer_params(b.id, 0, [peers[q][b.id][1].data_ptr() for q in range(world)])
+                for j in range(len(b.sizes)):
+                    R.ratel_register_peer_grads(b.id, j, [peers[q][b.id][j][0].data_ptr() for q in range(world)],
+                                                1.0 / world)
+                    R.ratel_register_peer_params(b.id, j, [peers[q][b.id][j][1].data_ptr() for q in range(world)])
         s = torch.cuda.Stream(device=dev)
         norms = []
         for t in range(1, STEPS + 1):
             with torch.cuda.stream(s):              # this rank's "backward"
                 for b in blocks:
-                    n = b.sizes[0]
-                    g = rank_grad(n, t, b.id, rank) if fused else synth.grad16(n, step=t, block=b.id)
-                    b.g16[0][:n].copy_(u16_to_torch(g, dev))
+                    g = rank_grad(b.total, t, b.id, rank) if fused else synth.grad16(b.total, step=t, block=b.id)
+                    for j, gj in enumerate(_split(g, b.sizes)):
+                        b.g16[j][:b.sizes[j]].copy_(u16_to_torch(gj, dev))
             R.ratel_adam_step(HPK["lr"], HPK["beta1"], HPK["beta2"], HPK["eps"], HPK["weight_decay"], t)
             for b in reversed(blocks):              # decreasing index, as backward produces them
                 R.ratel_offload_grad_chunk(b.id, s)
@@ -113,22 +121,23 @@ def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q):
                 norms.append(R.ratel_get_grad_sumsq())
         out = []
         for b in blocks:
-            n = b.sizes[0]
-            beg, end = R.ratel_rank_slice(n, world, rank)
-            k = end - beg
-            cap = R.ratel_padded_numel(n, world)
-            out.append(dict(p32=b.master[0][:k].cpu().numpy(), m32=b.m[0][:k].cpu().numpy(),
-                            v32=b.v[0][:k].cpu().numpy(), p16=torch_to_u16(b.p16[0][:n]),
-                            pad_nonzero=int(torch.count_nonzero(b.p16[0][n:cap].view(torch.int16)))))
+            for j, n in enumerate(b.sizes):
+                beg, end = R.ratel_rank_slice(n, world, rank)
+                k = end - beg
+                cap = R.ratel_padded_numel(n, world)
+                out.append(dict(p32=b.master[j][:k].cpu().numpy(), m32=b.m[j][:k].cpu().numpy(),
+                                v32=b.v[j][:k].cpu().numpy(), p16=torch_to_u16(b.p16[j][:n]),
+                                pad_nonzero=int(torch.count_nonzero(b.p16[j][n:cap].view(torch.int16)))))
         # checkpoint resume: scramble P16, refresh from the masters, all-gathered
         for b in blocks:
-            b.p16[0].fill_(7.0)
+            for p16 in b.p16:
+                p16.fill_(7.0)
         torch.cuda.synchronize()
         dist.barrier()                              # nobody's refresh may land before a peer scrambled
         for b in blocks:
             R.ratel_refresh_params(b.id, s)
         s.synchronize()
-        refreshed = [torch_to_u16(b.p16[0][:b.sizes[0]]) for b in blocks]
+        refreshed = [torch_to_u16(b.p16[j][:n]) for b in blocks for j, n in enumerate(b.sizes)]
         res_q.put((rank, out, norms, refreshed))
     except BaseException as e:  # report, then let the parent fail
         res_q.put((rank, repr(e), None, None))
@@ -145,13 +154,14 @@ def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q):
             pass
 
 
-def _run(mode, pinned, clip):
+def _run(mode, pinned, clip, blocks_spec=BLOCKS):
     world, shared = _plan()
     ctx = torch.multiprocessing.get_context("spawn")
     chans = {(a, b): ctx.Queue() for a in range(world) for b in range(world) if a != b}
     res_q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, mode, pinned, clip, chans, res_q))
+    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, mode, pinned, clip, chans, res_q,
+                                                              blocks_spec))
              for r in range(world)]
     for p in procs:
         p.start()
@@ -170,23 +180,30 @@ def _run(mode, pinned, clip):
     return world, results
 
 
-def _refs(world, fused, clip):
-    refs = [oracle.Range.fresh(synth.theta0(n, block=i)) for i, n in enumerate(SIZES)]
+def _refs(world, fused, clip, blocks_spec=BLOCKS):
+    """Oracle ranges in (block, range) order; the inputs exactly as the
+    GpuBlocks draw them (one synth stream per block, split by range)."""
+    refs = [oracle.Range.fresh(t) for i, sz in enumerate(blocks_spec)
+            for t in _split(synth.theta0(sum(sz), block=i), sz)]
     sums = []
     for t in range(1, STEPS + 1):
         hp = oracle.hparams(step=t, **HPK)
         if fused:
-            S, _ = oracle.adam_step_dp(refs, [[rank_grad(n, t, i, q) for q in range(world)]
-                                              for i, n in enumerate(SIZES)], 1.0 / world, hp, max_grad_norm=clip)
+            per_rank = [[g for i, sz in enumerate(blocks_spec) for g in _split(rank_grad(sum(sz), t, i, q), sz)]
+                        for q in range(world)]
+            S, _ = oracle.adam_step_dp(refs, [[per_rank[q][k] for q in range(world)] for k in range(len(refs))],
+                                       1.0 / world, hp, max_grad_norm=clip)
         else:
-            S, _ = oracle.adam_step(refs, [synth.grad16(n, step=t, block=i) for i, n in enumerate(SIZES)], hp,
+            S, _ = oracle.adam_step(refs, [g for i, sz in enumerate(blocks_spec)
+                                           for g in _split(synth.grad16(sum(sz), step=t, block=i), sz)], hp,
                                     max_grad_norm=clip)
         sums.append(S)
     return refs, sums
 
 
 def _check(world, results, refs, sums, what):
-    for i, n in enumerate(SIZES):
+    n_all = sum(r.p32.size for r in refs)
+    for i in range(len(refs)):
         got = {k: np.concatenate([results[r][0][i][k] for r in range(world)]) for k in ("p32", "m32", "v32")}
         got["p16"] = results[0][0][i]["p16"]
         check_range(got, refs[i], own_rne=oracle.bf16_rne, what=f"{what} block {i}")
@@ -199,7 +216,7 @@ def _check(world, results, refs, sums, what):
         for r in range(world):   # the clip allreduce: one global norm on every rank (all ranks' slices)
             for t, S in enumerate(sums):
                 # both double sums of exact squares, in different orders: n * 2^-53 relative
-                assert abs(results[r][1][t] - S) <= sum(SIZES) * 2.0 ** -53 * S, (what, r, t, results[r][1][t], S)
+                assert abs(results[r][1][t] - S) <= n_all * 2.0 ** -53 * S, (what, r, t, results[r][1][t], S)
             assert results[r][1] == results[0][1]
 
 
@@ -210,8 +227,16 @@ def test_nccl_allgather_and_clip_vs_oracle(cuda_dev, pinned, clip):
     _check(world, results, refs, sums, f"nccl N={world} pinned={pinned} clip={clip}")
 
 
-@pytest.mark.parametrize("pinned,clip", [(False, 0.0), (True, 1e-3)])
-def test_nccl_fused_reduce_scatter_and_allgather_vs_oracle(cuda_dev, pinned, clip):
-    world, results = _run("fused", pinned, clip)
-    refs, sums = _refs(world, True, clip)
-    _check(world, results, refs, sums, f"fused N={world} pinned={pinned} clip={clip}")
+@pytest.mark.parametrize("pinned,clip,multi", [(False, 0.0, False), (True, 1e-3, False), (False, 0.0, True),
+                                               (True, 1e-3, True)])
+def test_nccl_fused_reduce_scatter_and_allgather_vs_oracle(cuda_dev, pinned, clip, multi):
+    spec = BLOCKS_MULTI if multi else BLOCKS
+    world, results = _run("fused", pinned, clip, spec)
+    refs, sums = _refs(world, True, clip, spec)
+    _check(world, results, refs, sums, f"fused N={world} pinned={pinned} clip={clip} multi={multi}")
+
+
+def test_nccl_allgather_multirange_vs_oracle(cuda_dev):
+    world, results = _run("plain", False, 1e-3, BLOCKS_MULTI)
+    refs, sums = _refs(world, False, 1e-3, BLOCKS_MULTI)
+    _check(world, results, refs, sums, f"nccl N={world} multi-range clip")
