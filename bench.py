@@ -1116,6 +1116,48 @@ def auto_blocks(args, world: int) -> int:
     return k
 
 
+NCCL_LOG_DIR = os.path.join(ROOT, "build", "nccl_logs")
+
+
+def nccl_log_env() -> None:
+    """Keep NCCL's communicator-init log (transports, channels, NVLS) without
+    letting N ranks' INFO lines interleave with rank 0's JSON line on stdout:
+    NCCL_DEBUG=INFO (INIT, GRAPH, NVLS) into one file per process; rank 0
+    summarises its own file in multi_gpu.nccl_init and on stderr."""
+    if "NCCL_DEBUG" in os.environ:
+        return
+    os.makedirs(NCCL_LOG_DIR, exist_ok=True)
+    os.environ["NCCL_DEBUG"] = "INFO"
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT,GRAPH,NVLS,ENV")
+    os.environ["NCCL_DEBUG_FILE"] = os.path.join(NCCL_LOG_DIR, "nccl.%h.%p.log")
+
+
+def nccl_init_summary() -> dict | None:
+    """Key lines of this process's NCCL log: version, transports per peer,
+    NVLS / CollNet state, ring/tree channel counts, communicator sizes."""
+    path = os.environ.get("NCCL_DEBUG_FILE", "")
+    if not path:
+        return None
+    path = path.replace("%p", str(os.getpid()))
+    import glob
+    import socket
+    cands = glob.glob(path.replace("%h", "*"))
+    if not cands:
+        return {"log": path, "lines": []}
+    keys = ("NCCL version", "via P2P", "via NET", "via SHM", "NVLS", "nvls", "CollNet", "Channel 00",
+            "Init COMPLETE", "comm 0x", "Connected all rings", "Connected all trees", "NCCL_")
+    out = []
+    with open(cands[0], errors="replace") as f:
+        for line in f:
+            if any(k in line for k in keys):
+                out.append(line.strip()[:200])
+            if len(out) >= 40:
+                break
+    for line in out[:12]:
+        print("nccl:", line, file=sys.stderr)
+    return {"log": cands[0], "host": socket.gethostname(), "lines": out}
+
+
 def share_gpu_nccl_env(rank: int) -> None:
     """--share-gpu: NCCL refuses two ranks on one device of one host ("Duplicate
     GPU"); giving each rank its own NCCL host id makes them peers on different
@@ -1194,6 +1236,8 @@ def main():
         return
     if args.share_gpu and world > 1:
         share_gpu_nccl_env(rank)
+    if world > 1 and not args.sim_comm_none:
+        nccl_log_env()
 
     import torch
     import paper_conf_icde_liaosyxcyww25_b200 as R
@@ -1347,6 +1391,7 @@ def main():
                                           "step_over_max_bound": (ms / args.steps) / (1e3 * max(t_hbm, t_nv))}
                 multi = {"nccl_allgather": probes, "host_link": host_link_probe_all_ranks(torch, dev, world),
                          "own_params_max_rank": own_max,
+                         "nccl_init": nccl_init_summary() if rank == 0 else None,
                          "transport": ("loopback sockets, all ranks on one GPU (--share-gpu test mode)"
                                        if args.share_gpu else "NCCL over NVLink/NVSwitch")}
             except Exception as ex:  # report, do not hide

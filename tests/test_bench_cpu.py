@@ -102,3 +102,37 @@ def test_reference_arm_reports_the_sample_it_timed():
     for k in ("cpu_model", "numa_nodes", "sockets"):
         assert k in cb
     assert line["full_workload_ms_per_step_extrapolated"] > line["ms_per_step"]
+
+
+def test_auto_blocks_sizes_l_eff_to_the_box(monkeypatch):
+    """--blocks auto: host residencies keep all ranks' fp32 states within
+    85 % of MemAvailable (and P16 within 60 % of HBM); device residency fits
+    (12/N + 2) B/param into 95 % of HBM.  C2 at N=1 is the whole model."""
+    import argparse
+    sys.path.insert(0, ROOT)
+    import bench
+    monkeypatch.setattr(bench, "mem_available_bytes", lambda: 196 * 10 ** 9)
+    a = lambda shape, res: argparse.Namespace(shape=shape, residency=res)
+    assert bench.auto_blocks(a("13B", "device"), 1) == 41          # the whole C2 model (12.85B params)
+    assert bench.auto_blocks(a("70B", "host"), 1) == 17             # 0.85 * 196 GB / 9.66 GB per block
+    assert bench.auto_blocks(a("175B", "host"), 1) == 7             # 21.75 GB per block
+    assert bench.auto_blocks(a("70B", "host"), 8) == 17             # host RAM is shared by the ranks
+    n = bench.auto_blocks(a("30B", "device"), 8)
+    assert n == len(bench.model_blocks("30B"))                      # C3 fits at N = 8
+    for shape, res, w in (("70B", "host", 1), ("13B", "device", 1)):
+        k = bench.auto_blocks(a(shape, res), w)
+        sizes = bench.model_blocks(shape)[:k]
+        if res == "host":
+            assert 12 * sum(sizes) <= 0.85 * 196e9 < 12 * sum(bench.model_blocks(shape)[:k + 1])
+
+
+def test_nccl_log_summary(tmp_path, monkeypatch):
+    sys.path.insert(0, ROOT)
+    import bench
+    log = tmp_path / f"nccl.host.{os.getpid()}.log"
+    log.write_text("x NCCL INFO NCCL version 2.28.9+cuda12.9\nx NCCL INFO Channel 00/0 : 0[0] -> 1[1] via P2P/CUMEM\n"
+                   "irrelevant\nx NCCL INFO NVLS multicast support is available on dev 0\n")
+    monkeypatch.setenv("NCCL_DEBUG_FILE", str(tmp_path / "nccl.%h.%p.log"))
+    out = bench.nccl_init_summary()
+    assert out["log"] == str(log) and len(out["lines"]) == 3
+    assert any("via P2P" in line for line in out["lines"]) and any("NVLS" in line for line in out["lines"])
