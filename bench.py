@@ -1124,8 +1124,8 @@ def nccl_log_env() -> None:
     letting N ranks' INFO lines interleave with rank 0's JSON line on stdout:
     NCCL_DEBUG=INFO (INIT, GRAPH, NVLS) into one file per process; rank 0
     summarises its own file in multi_gpu.nccl_init and on stderr."""
-    if "NCCL_DEBUG" in os.environ:
-        return
+    if os.environ.get("NCCL_DEBUG_FILE"):
+        return                                   # the caller routes NCCL's log already
     os.makedirs(NCCL_LOG_DIR, exist_ok=True)
     os.environ["NCCL_DEBUG"] = "INFO"
     os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT,GRAPH,NVLS,ENV")
