@@ -286,6 +286,10 @@ def workload_config(args, world):
                                if args.sim_comm_none else "")) if world > 1 else "single GPU",
             "l2": "inputs larger than L2 (working set >> 126 MB)", "hyperparameters": HP,
             "max_grad_norm": args.clip, "update_streams": args.update_streams, "cta_tiles": args.cta_tiles,
+            **({"clip_schedule": "K2 (sum of g^2 partials, 2 B/param) at every hand-off, overlapping backward; "
+                                 "K3 + the norm allreduce and K1 of EVERY block only after the last hand-off "
+                                 "(the global norm needs all gradients): the update cannot overlap backward"}
+               if args.clip > 0 else {}),
             "k1_kernel": ["tma", "ldg", "ldg_lite"][args.k1_kernel], "staging": args.staging}
 
 
@@ -350,6 +354,7 @@ class Model:
                 p = symm_mem.empty(cap, dtype=torch.bfloat16, device=dev)
                 p.zero_()
                 hdl = symm_mem.rendezvous(p, dist.group.WORLD.group_name)
+                self.keep.append(hdl)          # the peer mappings live as long as the model
                 self.peer_ptrs.append(list(hdl.buffer_ptrs))
             else:
                 p = torch.zeros(cap, dtype=torch.bfloat16, device=dev)

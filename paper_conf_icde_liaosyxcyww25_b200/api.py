@@ -108,8 +108,9 @@ class _PeerArena:
             self.p16.zero_()
             self.g16.zero_()
             group = dist.group.WORLD.group_name
-            self.bases_p = list(symm_mem.rendezvous(self.p16, group).buffer_ptrs)
-            self.bases_g = list(symm_mem.rendezvous(self.g16, group).buffer_ptrs)
+            self.handles = (symm_mem.rendezvous(self.p16, group), symm_mem.rendezvous(self.g16, group))
+            self.bases_p = list(self.handles[0].buffer_ptrs)   # the handles stay referenced with the arena
+            self.bases_g = list(self.handles[1].buffer_ptrs)
         elif peer_memory == "ipc":
             from torch.multiprocessing.reductions import reduce_tensor
             self.p16 = torch.zeros(n, dtype=torch.bfloat16, device=dev)
