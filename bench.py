@@ -1214,7 +1214,8 @@ def main():
     ap.add_argument("--overlap-host-sweep", type=lambda x: [int(v) for v in x.split(",") if v],
                     default=[32768, 65536, 98304, 131072, 196608],
                     help="pinned-host per-tensor AGO overlap probe: tokens per step, comma-separated ('' disables)")
-    ap.add_argument("--overlap-host-blocks", type=int, default=8)
+    ap.add_argument("--overlap-host-blocks", type=int, default=16,
+                    help="13B-shape blocks of pinned-host states in the host overlap probe (16 = 5.0B params, 60 GB)")
     ap.add_argument("--arm", default="before", choices=["before", "after"],
                     help="arm before the hand-offs (AGO) or after the last one (deferred)")
     ap.add_argument("--cta-tiles", type=int, default=0, help="cfg.cta_tiles (0 = persistent update grid)")
