@@ -43,9 +43,13 @@ STEPS = 3
 HPK = dict(lr=1e-3, beta1=0.9, beta2=0.999, eps=1e-8, weight_decay=1e-2)
 
 
-def _plan():
+def _plan(world=None):
+    """(world, shared): one GPU per rank when the box has them, else every
+    rank on cuda:0 with its own NCCL host id."""
     n = torch.cuda.device_count()
-    return (min(n, 8), False) if n >= 2 else (2, True)
+    if world is None:
+        return (min(n, 8), False) if n >= 2 else (2, True)
+    return world, n < world
 
 
 def rank_grad(n, step, block, q):
@@ -154,8 +158,8 @@ def _rank_main(rank, world, shared, port, mode, pinned, clip, chans, res_q, bloc
             pass
 
 
-def _run(mode, pinned, clip, blocks_spec=BLOCKS):
-    world, shared = _plan()
+def _run(mode, pinned, clip, blocks_spec=BLOCKS, world=None):
+    world, shared = _plan(world)
     ctx = torch.multiprocessing.get_context("spawn")
     chans = {(a, b): ctx.Queue() for a in range(world) for b in range(world) if a != b}
     res_q = ctx.Queue()
@@ -234,6 +238,17 @@ def test_nccl_fused_reduce_scatter_and_allgather_vs_oracle(cuda_dev, pinned, cli
     world, results = _run("fused", pinned, clip, spec)
     refs, sums = _refs(world, True, clip, spec)
     _check(world, results, refs, sums, f"fused N={world} pinned={pinned} clip={clip} multi={multi}")
+
+
+@pytest.mark.parametrize("world", [4, 8])
+def test_nccl_allgather_and_fused_at_4_and_8_ranks(cuda_dev, world):
+    """N = 4 and 8 ranks: slices padded to 8N elements (ragged tails, a
+    24-element range with empty slices on most ranks), the in-place NCCL
+    all-gather with clip, then the fused path, all on a real communicator."""
+    for mode, clip in (("plain", 1e-3), ("fused", 0.0)):
+        w, results = _run(mode, False, clip, BLOCKS, world=world)
+        refs, sums = _refs(w, mode == "fused", clip, BLOCKS)
+        _check(w, results, refs, sums, f"{mode} N={w} clip={clip}")
 
 
 def test_nccl_allgather_multirange_vs_oracle(cuda_dev):
