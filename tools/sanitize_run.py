@@ -2,7 +2,8 @@
 racecheck, synccheck): C1-sized ragged blocks, a capped grid so every CTA
 cycles the TMA stage ring, clip mode, a pinned-host block, the register-staged
 LDG / LDG_LITE kernels, a non-persistent grid (cta_tiles), zero-copy staging
-and the fused-reduction kernels (K1-RS, K2-RS) at world 1."""
+and the fused-reduction kernels (K1-RS, K2-RS) at world 1; every run ends with
+ratel_refresh_params (refresh_p16_kernel over device and pinned-host masters)."""
 import os
 import sys
 
@@ -31,6 +32,8 @@ def run(max_ctas, clip, pinned, rs_scale=None, **cfg):
             for b in reversed(blocks):
                 R.ratel_offload_grad_chunk(b.id, None)
             R.ratel_sync(None)
+        for b in blocks:                       # P16 rebuilt from the masters (refresh_p16_kernel)
+            R.ratel_refresh_params(b.id, None)
 
 
 if __name__ == "__main__":
