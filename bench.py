@@ -794,6 +794,44 @@ def nccl_allgather_probe(torch, dev, world, counts, reps=5):
     return out
 
 
+def nccl_allreduce_latency_us(torch, dev, world, reps=50):
+    """Latency of the clip's 8-byte fp64 allreduce (X1) on this world:
+    median of `reps` back-to-back single calls, CUDA events, max over ranks."""
+    import torch.distributed as dist
+    x = torch.zeros(1, dtype=torch.float64, device=dev)
+    for _ in range(5):
+        dist.all_reduce(x)
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        dist.all_reduce(x)
+        e1.record()
+        e1.synchronize()
+        ts.append(e0.elapsed_time(e1) * 1e3)
+    return max_over_ranks(torch, sorted(ts)[len(ts) // 2], world, dev)
+
+
+def p16_identical_across_ranks(torch, dev, world, p16s) -> bool:
+    """Every rank holds the same gathered P16 (bitwise
+    equality of all ranks' bf16): two position-weighted int64 checksums over
+    every block's P16 words, compared across ranks."""
+    import torch.distributed as dist
+    C = 1 << 24
+    w = (torch.arange(C, device=dev, dtype=torch.int64) % 65521) + 1
+    acc = torch.zeros(2, dtype=torch.int64, device=dev)
+    for p in p16s:
+        words = p.view(torch.int16)
+        for k in range(0, words.numel(), C):
+            x = words[k:k + C].to(torch.int64)
+            acc[0] += x.sum()
+            acc[1] += (x * w[:x.numel()]).sum()
+    allv = [torch.zeros_like(acc) for _ in range(world)]
+    dist.all_gather(allv, acc)
+    return all(torch.equal(allv[0], v) for v in allv[1:])
+
+
 def host_link_probe_all_ranks(torch, dev, world):
     """The duplex host-link probe run in every rank at once (started behind a
     barrier): per-rank and aggregate GB/s -- the pinned-host roofline at this
@@ -1396,6 +1434,8 @@ def main():
                                           "max": 1e3 * max(t_hbm, t_nv),
                                           "step_over_max_bound": (ms / args.steps) / (1e3 * max(t_hbm, t_nv))}
                 multi = {"nccl_allgather": probes, "host_link": host_link_probe_all_ranks(torch, dev, world),
+                         "nccl_allreduce_8B_latency_us": nccl_allreduce_latency_us(torch, dev, world),
+                         "p16_identical_across_ranks": p16_identical_across_ranks(torch, dev, world, model.p16),
                          "own_params_max_rank": own_max,
                          "nccl_init": nccl_init_summary() if rank == 0 else None,
                          "transport": ("loopback sockets, all ranks on one GPU (--share-gpu test mode)"
