@@ -1466,7 +1466,8 @@ def main():
             e2e = e2e_host
         if args.residency != "device":      # the bound is off-device: report that roofline, K1 beside it
             try:
-                roof = offdevice_roofline(args, torch, dev, own * args.steps / (ms / 1e3), roof)
+                nv = {k: roof[k] for k in ("nvlink", "step_bounds_ms") if k in roof}
+                roof = dict(offdevice_roofline(args, torch, dev, own * args.steps / (ms / 1e3), roof), **nv)
             except Exception as ex:  # report, do not hide
                 roof = dict(roof, offdevice_error=repr(ex)[:300])
 
