@@ -1858,6 +1858,10 @@ int ratel_refresh_params(int block_id, void* stream) {
   if (block_id < 0 || block_id >= RATEL_MAX_BLOCKS || !G.blocks[block_id].registered)
     return set_error(RATEL_ESTATE, "ratel_refresh_params: block %d is not registered", block_id);
   Block& B = G.blocks[block_id];
+  if (B.residency == RATEL_SSD)  // every non-empty slice needs its state file (no side effects on ESTATE)
+    for (size_t i = 0; i < B.ranges.size(); ++i)
+      if (B.ssd[i].fd < 0 && B.slices[i].end > B.slices[i].begin)
+        return set_error(RATEL_ESTATE, "ratel_refresh_params: block %d range %zu has no SSD file", block_id, i);
   const cudaStream_t cs = static_cast<cudaStream_t>(stream);
   // after whatever the caller enqueued (e.g. restored states), and after every
   // earlier update (s_opt is ordered after all of them by ratel_sync)
@@ -1890,10 +1894,6 @@ int ratel_refresh_params(int block_id, void* stream) {
       return sticky_fail(RATEL_ENOMEM, "ratel_refresh_params: staging cudaHostAlloc failed");
     }
     const Block::SsdRange& f = B.ssd[i];
-    if (f.fd < 0) {
-      rc = set_error(RATEL_ESTATE, "ratel_refresh_params: block %d range %zu has no SSD file", block_id, i);
-      break;
-    }
     for (uint64_t off = 0; off < n && rc == RATEL_OK; off += T) {
       const uint64_t len = std::min<uint64_t>(T, n - off);
       const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
