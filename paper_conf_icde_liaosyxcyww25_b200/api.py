@@ -149,7 +149,7 @@ class _Range:
         cap = R.ratel_padded_numel(self.numel, world)
         beg, end = R.ratel_rank_slice(self.numel, world, rank)
         self.peer_p16 = self.peer_g16 = None
-        if arena is not None:   # world > 1, data parallel: symmetric memory
+        if arena is not None:   # world > 1, data parallel: memory every rank maps
             self.p16, self.g16, self.peer_p16, self.peer_g16 = arena.take(cap)
         else:
             self.p16 = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
@@ -173,8 +173,7 @@ class _Range:
             self.master, self.m, self.v = mk(), mk(), mk()
             if end > beg:
                 self.master[:end - beg].copy_(flat32[beg:end])
-        self.p16[:self.numel].copy_(flat32.to(torch.bfloat16))
-        off = 0
+        off = 0                     # P16 is built from the masters by the library (ratel_refresh_params)
         for p in params:  # parameters become views of the flat buffers
             k = p.numel()
             p.data = self.p16[off:off + k].view(p.shape)
@@ -338,6 +337,13 @@ class Ratel_Optimizer:
                 for i, r in enumerate(ranges):
                     R.ratel_register_peer_grads(bid, i, r.peer_g16, 1.0 / world)
                     R.ratel_register_peer_params(bid, i, r.peer_p16)
+        # the working copy P16 = bf16_rne(master), built by the library (the
+        # update's own conversion) and all-gathered across ranks -- collective
+        s = torch.cuda.current_stream()
+        for bid in self.block_ids:
+            for lid in self._lib_ids[bid]:
+                R.ratel_refresh_params(lid, s)
+        torch.cuda.synchronize()
         self._pending = {}
         self._handed = set()
         self._hooks = []
