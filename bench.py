@@ -322,10 +322,13 @@ class PinnedArena:
 
 class Model:
     """Synthetic model states of one rank: per block one flat range.
-    symm=True allocates P16 in torch symmetric memory (peer-mapped) for the
-    fused update + all-gather (ratel_register_peer_params)."""
+    symm=True allocates P16 in memory every rank maps, for the fused update +
+    all-gather (ratel_register_peer_params): torch symmetric memory, or with
+    peer_memory="ipc" plain allocations opened through CUDA IPC handles (ranks
+    sharing a GPU, where symmetric memory refuses)."""
 
-    def __init__(self, R, torch, dev, sizes, world, rank, residency, grad_ring=2, pin_grads=False, symm=False):
+    def __init__(self, R, torch, dev, sizes, world, rank, residency, grad_ring=2, pin_grads=False, symm=False,
+                 peer_memory="symm"):
         self.sizes = sizes
         self.ranges = []
         self.keep = []
@@ -348,7 +351,20 @@ class Model:
             cap = R.ratel_padded_numel(n, world)
             beg, end = R.ratel_rank_slice(n, world, rank)
             s = max(end - beg, 8)
-            if symm:
+            if symm and peer_memory == "ipc":
+                import torch.distributed as dist
+                from torch.multiprocessing.reductions import reduce_tensor
+                p = torch.zeros(cap, dtype=torch.bfloat16, device=dev)
+                torch.cuda.synchronize()
+                allh = [None] * world
+                dist.all_gather_object(allh, reduce_tensor(p))
+                ptrs = []
+                for q, h in enumerate(allh):
+                    t = p if q == rank else h[0](*h[1])
+                    self.keep.append(t)            # the peer mappings live as long as the model
+                    ptrs.append(t.data_ptr())
+                self.peer_ptrs.append(ptrs)
+            elif symm:
                 import torch.distributed as dist
                 import torch.distributed._symmetric_memory as symm_mem
                 p = symm_mem.empty(cap, dtype=torch.bfloat16, device=dev)
@@ -1323,7 +1339,7 @@ def main():
     try:
         fused = args.fused_allgather and world > 1 and not SIM_COMM_NONE
         model = Model(R, torch, dev, sizes, world, rank, "device" if args.residency == "device" else "host",
-                      symm=fused)
+                      symm=fused, peer_memory="ipc" if args.share_gpu else "symm")
         res = {"host": R.RATEL_PINNED_HOST, "hostcompute": R.RATEL_HOST_COMPUTE}.get(args.residency, R.RATEL_DEVICE)
         hybrid = args.residency == "hybrid"
         if hybrid and world > 1:
