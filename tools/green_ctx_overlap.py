@@ -35,6 +35,8 @@ def main():
     ap.add_argument("--tokens", type=int, nargs="+", default=[8192, 32768])
     ap.add_argument("--sms", type=int, nargs="+", default=[8, 16, 32])
     ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--residency", default="device", choices=["device", "host"],
+                    help="host: pinned-host states, per-tensor hand-off (the tile updates capped at k CTAs)")
     args = ap.parse_args()
     from torch.cuda.green_contexts import SUPPORTED, GreenContext
     if not SUPPORTED:
@@ -47,15 +49,29 @@ def main():
     sizes = bench.model_blocks("13B", with_embedding=False)[:args.blocks]
     cfg = R.ratel_default_config()
     R.ratel_init(0, 0, 1, None, cfg)
-    model = bench.Model(R, torch, dev, sizes, 1, 0, "device", grad_ring=3)
+    model = bench.Model(R, torch, dev, sizes, 1, 0, args.residency, grad_ring=3)
     R.ratel_finalize()
+    host = args.residency == "host"
+    K = 4 if host else 1                # per-tensor units for the pinned-host path
+    units = {}
+    for b, n in enumerate(sizes):
+        if not host:
+            units[b] = [model.ranges[b]]
+            continue
+        r0, offs, off = model.ranges[b], [], 0
+        for (o, i) in bench.linears(h):
+            offs.append([off, o * i])
+            off += o * i
+        offs[-1][1] += n - off
+        units[b] = [R.ratel_range(r0.param_bf16 + 2 * o, r0.grad_bf16 + 2 * o, 0, r0.master + 4 * o,
+                                  r0.exp_avg + 4 * o, r0.exp_avg_sq + 4 * o, ln, 1) for o, ln in offs]
     order = list(reversed(range(len(sizes))))
     nr = 3
     relay = torch.cuda.Stream()         # primary-context hand-off stream
     relay2 = torch.cuda.Stream()        # primary-context ring-recycling stream
     out = []
     for T in args.tokens:
-        bw = bench.SynthBackward(dev, h, T, model.p16, model.grad_ring, 0, chunk=16384)
+        bw = bench.SynthBackward(dev, h, T, model.p16, model.grad_ring, 0, chunk=65536 if host else 16384)
         for k in [0] + list(args.sms):
             gc = GreenContext.create(nsm - k, 0) if k > 0 else None
             cfg = R.ratel_default_config()
@@ -63,7 +79,8 @@ def main():
             R.ratel_init(0, 0, 1, None, cfg)
             try:
                 for b in range(len(sizes)):
-                    R.ratel_register_block(b, [model.ranges[b]], R.RATEL_DEVICE)
+                    for j, r in enumerate(units[b]):
+                        R.ratel_register_block(b * K + j, [r], R.RATEL_PINNED_HOST if host else R.RATEL_DEVICE)
                 t = [1]
 
                 def arm():
@@ -93,28 +110,40 @@ def main():
                     arm()
                     for j, b in enumerate(order):
                         if j >= nr:                       # the ring slot's previous update ran
-                            R.ratel_block_wait(b + nr, relay2)
+                            for q in range(K):
+                                R.ratel_block_wait((b + nr) * K + q, relay2)
                             ev_free = torch.cuda.Event()
                             ev_free.record(relay2)
                         else:
                             ev_free = None
 
                         def f(s, b=b, ev_free=ev_free):
+                            # every library call happens after the context is popped: the
+                            # per-linear events are collected here and relayed below (the
+                            # GEMMs are already enqueued, so the GPU timeline is the same)
                             if ev_free is not None:
                                 s.wait_event(ev_free)
+                            evs = []
+
+                            def on_linear(q, s=s, b=b):
+                                ev = torch.cuda.Event()
+                                ev.record(s)
+                                evs.append((b * K + q, ev))
                             with torch.cuda.stream(s):
-                                bw.block(b, b % nr)
+                                bw.block(b, b % nr, on_linear=on_linear if host else None)
                             ev = torch.cuda.Event()
                             ev.record(s)
-                            return ev
-                        relay.wait_event(in_green(f))
-                        R.ratel_offload_grad_chunk(b, relay)
+                            return evs or [(b, ev)]
+                        for uid, ev in in_green(f):
+                            relay.wait_event(ev)
+                            R.ratel_offload_grad_chunk(uid, relay)
                     R.ratel_sync(relay)
 
                 def opt():
                     arm()
                     for b in order:
-                        R.ratel_offload_grad_chunk(b, relay)
+                        for q in range(K):
+                            R.ratel_offload_grad_chunk(b * K + q, relay)
                     R.ratel_sync(relay)
 
                 def timed(fn):
@@ -137,7 +166,8 @@ def main():
                     b_runs.append(timed(bwd_only))
                 base = [0.5 * (b_runs[i] + b_runs[i + 1]) for i in range(args.reps)]
                 exp = sorted(a - b for a, b in zip(a_runs, base))
-                row = {"tokens": T, "green_sms_backward": nsm - k if k else nsm, "update_ctas": k or "all",
+                row = {"residency": args.residency, "tokens": T, "green_sms_backward": nsm - k if k else nsm,
+                       "update_ctas": k or "all",
                        "blocks": len(sizes), "backward_ms": sorted(base)[len(base) // 2], "optimizer_alone_ms": t_opt,
                        "ago_ms": sorted(a_runs)[len(a_runs) // 2], "exposed_ms": exp[len(exp) // 2],
                        "exposed_ms_spread": [exp[0], exp[-1]], "backward_ms_runs": b_runs}
