@@ -57,7 +57,7 @@ def _flat_ranges(model):
     return out
 
 
-def _rank_main(rank, world, shared, port, res_q, peer_memory):
+def _rank_main(rank, world, shared, port, res_q, peer_memory, data_parallel="fused"):
     if shared:
         os.environ["NCCL_HOSTID"] = f"ratel-api-rank{rank}"
         os.environ["NCCL_SOCKET_IFNAME"] = "lo"
@@ -84,12 +84,13 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
         model = torch.nn.Sequential(*[Block(D) for _ in range(NB)]).to(dev)
         init = _flat_ranges(model)
         gen = torch.Generator(device=dev)
-        gen.manual_seed(100 + rank)                        # a different micro-batch per rank
+        # fused: a different micro-batch per rank; reduced: the same one (identical grads, R11)
+        gen.manual_seed(100 + (rank if data_parallel == "fused" else 0))
         xs = [torch.randn(32, D, device=dev, dtype=torch.bfloat16, generator=gen) for _ in range(STEPS + 2)]
         with Ratel_init():
             opt = Ratel_Optimizer([list(b.parameters()) for b in model], lr=HPK["lr"],
                                   betas=(HPK["beta1"], HPK["beta2"]), eps=HPK["eps"],
-                                  weight_decay=HPK["weight_decay"], data_parallel="fused",
+                                  weight_decay=HPK["weight_decay"], data_parallel=data_parallel,
                                   peer_memory=peer_memory)
             Ratel_hook(opt)
             ranges = [r for rs in opt.blocks for r in rs]
@@ -100,7 +101,7 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
                 torch.cuda.synchronize()
                 local_grads.append([r.g16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16)
                                     for r in ranges])
-                if t == 0:   # what this rank sees through its mapping of the peer's G16
+                if t == 0 and data_parallel == "fused":   # this rank's view of the peer's G16
                     dist.barrier()
                     q = 1 - rank
                     peer_view = []
@@ -131,7 +132,8 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory):
             reloaded = [r.p16[:r.numel].view(torch.int16).cpu().numpy().view(np.uint16) for r in ranges]
             opt.remove_hooks()
             del opt
-        res_q.put((rank, init, local_grads, out, reloaded, peer_view, handoffs))
+        res_q.put((rank, init, local_grads, out, reloaded, peer_view if data_parallel == "fused" else None,
+                   handoffs))
     except BaseException as e:
         res_q.put((rank, repr(e), None, None, None, None, None))
         raise
@@ -168,18 +170,22 @@ def _diagnose(init, res, world, k, got):
     return out
 
 
-@pytest.mark.parametrize("peer_memory", ["ipc", "symm"])
-def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
+@pytest.mark.parametrize("peer_memory,data_parallel", [("ipc", "fused"), ("symm", "fused"), ("symm", "reduced")])
+def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_parallel):
     """peer_memory="symm" (torch symmetric memory) needs a GPU per rank; on a
-    one-GPU box only the CUDA-IPC mapping runs."""
+    one-GPU box only the CUDA-IPC mapping runs.  data_parallel="reduced": both
+    ranks see the same micro-batch (identical gradients, R11), the library only
+    all-gathers P16 over NCCL -- the mean of identical gradients is the same
+    step, so the same oracle check applies."""
     n = torch.cuda.device_count()
     world, shared = (2, n < 2)
-    if shared and peer_memory == "symm":
+    if shared and peer_memory == "symm" and data_parallel == "fused":
         pytest.skip("torch symmetric memory refuses ranks that share a GPU")
     ctx = torch.multiprocessing.get_context("spawn")
     res_q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, res_q, peer_memory)) for r in range(world)]
+    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, res_q, peer_memory, data_parallel))
+             for r in range(world)]
     for p in procs:
         p.start()
     res = {}
@@ -197,7 +203,7 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
     init = res[0][0]
     # the hand-off order (each hand-off is a barrier on the library's communicator) is the same on both ranks
     assert [h[0] for h in res[0][5]] == [h[0] for h in res[1][5]], (res[0][5], res[1][5])
-    for q in range(world):   # the mapping of the peer's G16 shows the peer's gradient
+    for q in range(world if data_parallel == "fused" else 0):   # the mapping of the peer's G16
         for k in range(len(init)):
             assert np.array_equal(res[q][4][k], res[1 - q][1][0][k]), ("peer view", q, k)
     for k in range(len(init)):
@@ -205,7 +211,8 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory):
     wd = [1, 0] * NB                                           # weights decay, biases / LN do not
     refs = [oracle.Range.fresh(a.astype(np.float32), wd[k]) for k, a in enumerate(init)]
     for t in range(STEPS):
-        assert not all(np.array_equal(res[0][1][t][k], res[1][1][t][k]) for k in range(len(refs)))
+        same = all(np.array_equal(res[0][1][t][k], res[1][1][t][k]) for k in range(len(refs)))
+        assert same == (data_parallel == "reduced"), t
         oracle.adam_step_dp(refs, [[res[q][1][t][k] for q in range(world)] for k in range(len(refs))],
                             1.0 / world, oracle.hparams(step=t + 1, **HPK))
     for k, ref in enumerate(refs):
