@@ -1261,7 +1261,7 @@ def main():
     ap.add_argument("--share-gpu", action="store_true",
                     help="test mode: every rank on cuda:0 with real NCCL (each rank its own NCCL host id, "
                          "loopback sockets); numbers are plumbing, not a scaling result")
-    ap.add_argument("--overlap-sweep", type=lambda x: [int(v) for v in x.split(",") if v], default=[2048, 8192, 32768, 65536],
+    ap.add_argument("--overlap-sweep", type=lambda x: [int(v) for v in x.split(",") if v], default=[1024, 2048, 8192, 32768, 65536],
                     help="device-resident AGO vs deferred overlap sweep: tokens per step, comma-separated "
                          "('' disables)")
     ap.add_argument("--overlap-reps", type=int, default=3, help="alternating repetitions per overlap point")
