@@ -62,6 +62,8 @@ MUTANTS = {
     "m_bar_drops_1_minus_beta1": ("(1.0 - hp->beta1) * fabs(g_used);", "fabs(g_used);"),
     "m_bar_uses_beta2": ("m_bar[i] = hp->beta1 * m_bar[i] + (1.0 - hp->beta1) * fabs(g_used);",
                          "m_bar[i] = hp->beta2 * m_bar[i] + (1.0 - hp->beta2) * fabs(g_used);"),
+    "scales_ignore_clip": ("update_scales(i, gu, ad, apply_wd, hp, theta_bar, m_bar);\n  }\n}\n\n/* Same update",
+                           "update_scales(i, gu / coef, ad, apply_wd, hp, theta_bar, m_bar);\n  }\n}\n\n/* Same update"),
     "m_bar_l2_from_raw_grad": [("double th = *theta;", "double th = *theta;\n  *g_used = g;"),
                                ("  *g_used = g;\n  return fabs(delta);", "  return fabs(delta);")],
 }
@@ -150,6 +152,12 @@ def _pins_pass():
             return False
         exp = np.array([0.01, 0.02, 0.03, 0.0], np.float32).astype(np.float64) + 5 * lr * c / (c + eps)
         if not np.all(np.abs(r.theta_bar - exp) <= 2.0 ** -18 * exp):
+            return False
+        # scales under the clip: built from the clipped gradient coef * g
+        r = oracle.Range.fresh(th0)
+        _, coef = oracle.adam_step([r], [g], oracle.hparams(step=1), max_grad_norm=1e-4)
+        gp = coef * synth.bf16_bits_to_f32(g).astype(np.float64)
+        if not (coef < 1 and np.all(np.abs(r.m_bar - 0.1 * np.abs(gp)) <= 1e-12 * np.abs(gp))):
             return False
         # torch.optim.AdamW, 10 steps, fp32 storage emulated (R13 bound 1e-6)
         from tests.tolerance import check_range

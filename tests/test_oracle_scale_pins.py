@@ -196,3 +196,22 @@ def test_scales_mpmath_trace(mode):
                 ex = float(ex)
                 assert abs(float(got) - ex) <= 0.5 * float(np.spacing(np.float32(abs(ex)))) * (1 + 1e-6) + 1e-300, \
                     (t, i, float(got), ex)
+
+
+def test_scales_step1_with_clip_use_the_clipped_gradient():
+    """With the global-norm clip the update sees g' = coef * g (R9, torch's
+    clip_grad_norm_), so the scales are built from it: m_bar_1 = (1-b1)|g'|,
+    theta_bar_1 = d|theta_0| + lr|g'|/(|g'|+eps), coef from the float64 norm."""
+    import torch
+    n, max_norm = 4096, 1e-4
+    th0 = synth.theta0(n, block=47)
+    g = synth.grad16(n, step=1, block=47)
+    r = oracle.Range.fresh(th0)
+    S, coef = oracle.adam_step([r], [g], oracle.hparams(step=1), max_grad_norm=max_norm)
+    norm = float(torch.linalg.vector_norm(torch.from_numpy(_g(g))))
+    c = max_norm / (norm + 1e-6)
+    assert 0 < c < 1 and abs(coef - c) <= 1e-12 * c
+    gp = c * _g(g)
+    assert close(r.m_bar, (1 - B1) * np.abs(gp), 1e-12)
+    exp = (1 - LR * 1e-2) * np.abs(th0.astype(np.float64)) + LR * np.abs(gp) / (np.abs(gp) + EPS)
+    assert close(r.theta_bar, exp, 2.0 ** -21)
