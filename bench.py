@@ -654,6 +654,7 @@ def overlap_host_probe(args, R, torch, dev, dev_index, energy=None):
     order = list(reversed(range(len(sizes))))
     P = sum(sizes)
     out = {}
+    bw0 = None
     # one set of activations (<= 64K tokens per GEMM chunk) serves every T of the sweep
     bw0 = SynthBackward(dev, h, max(args.overlap_host_sweep), model.p16, model.grad_ring, 0, chunk=65536)
     # settle the GPU at its thermal/power operating point first: measured, the same
