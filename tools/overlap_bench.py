@@ -131,6 +131,7 @@ def run(args):
             else:
                 if schedule != "deferred":
                     arm()
+                held = []                                       # --group: blocks not yet handed off
                 for j, b in enumerate(order):
                     if schedule != "deferred" and j >= args.ring:
                         wait_all(b + args.ring, hi)             # ring slot free
@@ -138,7 +139,11 @@ def run(args):
                         bw.block(b, b % args.ring, on_linear=lambda k, b=b: handoff_unit(b, k, hi))
                     else:
                         bw.block(b, b % args.ring)
-                        handoff_unit(b, 0, hi)
+                        held.append(b)
+                        if len(held) >= args.group or j == len(order) - 1:
+                            for x in held:                      # a burst of hand-offs: one update phase
+                                handoff_unit(x, 0, hi)
+                            held = []
                     if timeline:
                         tl["g"][b] = torch.cuda.Event(enable_timing=True)
                         tl["g"][b].record(hi)
@@ -216,6 +221,7 @@ def run(args):
             row = {"residency": args.residency + (f" {args.hybrid_gpu_frac}" if hybrid else ""),
                    "host_threads": args.host_threads, "granularity": args.granularity, "cta_tiles": args.cta_tiles,
                    "k1_kernel": args.k1_kernel, "bwd_priority": args.bwd_priority, "ring": args.ring,
+                   "group": args.group,
                    "tile_elems": args.tile_elems, "zero_copy": bool(args.zero_copy),
                    "tokens": tokens, "max_ctas": mc,
                    "carveout": bool(args.carveout),
@@ -250,6 +256,9 @@ if __name__ == "__main__":
     ap.add_argument("--max-ctas", type=int, nargs="+", default=[0, 32])
     ap.add_argument("--schedules", nargs="+", default=["bwd", "opt", "ago", "deferred", "naive"])
     ap.add_argument("--ring", type=int, default=3)
+    ap.add_argument("--group", type=int, default=1,
+                    help="hand blocks off in bursts of this many (fewer GEMM/update interleave points; "
+                         "needs --ring >= 2 * group)")
     ap.add_argument("--steps", type=int, default=3)
     ap.add_argument("--warmup", type=int, default=1)
     ap.add_argument("--timeline", action="store_true", help="per-block grad-ready / update-done times")
