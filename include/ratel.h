@@ -158,6 +158,13 @@ typedef enum { RATEL_UPDATE_TMA = 0, RATEL_UPDATE_LDG = 1, RATEL_UPDATE_LDG_LITE
  * tensor i-1", at tile granularity. */
 typedef enum { RATEL_SSD_DUPLEX = 0, RATEL_SSD_SIMPLEX = 1 } ratel_ssd_schedule;
 
+/* SSD tier I/O method.  PREAD: each thread moves a tile's three arrays with
+ * blocking pread/pwrite, one request at a time.  URING: each thread owns an
+ * io_uring (raw syscalls) and keeps up to 32 requests of <= 4 MiB in flight
+ * (queue depth > 1, what an NVMe needs to reach its bandwidth); a kernel that
+ * refuses io_uring makes the first SSD registration fail with RATEL_EIO. */
+typedef enum { RATEL_SSD_IO_PREAD = 0, RATEL_SSD_IO_URING = 1 } ratel_ssd_io;
+
 typedef struct {
   int mode;               /* ratel_mode; default RATEL_ADAMW */
   double max_grad_norm;   /* > 0 enables the global L2-norm clip (torch clip_grad_norm_); default 0 */
@@ -181,6 +188,8 @@ typedef struct {
                              default RATEL_UPDATE_TMA.  Results are identical. */
   int ssd_schedule;       /* ratel_ssd_schedule: RATEL_SSD* tiers; default RATEL_SSD_DUPLEX.  Results are
                              identical. */
+  int ssd_io;             /* ratel_ssd_io: how the SSD tier's threads move tiles; default RATEL_SSD_IO_PREAD.
+                             Results are identical. */
 } ratel_config;
 
 /* One contiguous parameter range of a block (a flat tensor, or a block's

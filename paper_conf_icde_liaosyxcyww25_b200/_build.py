@@ -16,7 +16,7 @@ CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libratel.so")
 SOURCES = ["ratel_runtime.cu", "ratel_gen.cu", "ratel_host_adam.cpp", "ratel_plan.cpp"]
-HEADERS = ["ratel_kernels.cuh", "ratel_bf16.cuh", "nccl_dl.h", "ratel_host_adam.h", "ratel_plan_impl.h"]
+HEADERS = ["ratel_kernels.cuh", "ratel_bf16.cuh", "nccl_dl.h", "ratel_host_adam.h", "ratel_plan_impl.h", "ratel_uring.h"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

@@ -39,6 +39,7 @@
 #include "ratel.h"
 #include "ratel_host_adam.h"
 #include "ratel_plan_impl.h"
+#include "ratel_uring.h"
 #include "ratel_kernels.cuh"
 
 namespace {
@@ -137,6 +138,7 @@ struct SsdEngine {
   uint64_t jobs_in = 0, jobs_out = 0, tiles_in = 0, tiles_out = 0;
   int err = 0;
   std::string msg;
+  IoRing rd_ring, wr_ring;   // RATEL_SSD_IO_URING: the reader's and the writer's io_uring
   float* h_ring = nullptr;  // pinned: depth x {theta, m, v} x tile
   float* d_ring = nullptr;  // device: the same shape
   cudaStream_t s_in = nullptr, s_k = nullptr, s_out = nullptr;
@@ -727,6 +729,23 @@ int io_full(bool rd, int fd, void* buf, uint64_t bytes, uint64_t off, std::strin
   return RATEL_OK;
 }
 
+// The three arrays (theta, m, v) of one staged tile: file <-> pinned staging,
+// by pread/pwrite one request at a time or through the thread's io_uring.
+int io_tile(SsdEngine& E, IoRing& ring, bool rd, int fd, float* h, uint64_t T, uint64_t bytes, uint64_t foff,
+            uint64_t stride, std::string& msg) {
+  if (G.cfg.ssd_io == RATEL_SSD_IO_URING) {
+    std::vector<IoRing::Req> reqs;
+    for (int a = 0; a < 3; ++a) reqs.push_back({h + a * T, bytes, foff + a * stride});
+    return ring.transfer(rd, fd, reqs, msg) == 0 ? RATEL_OK : RATEL_EIO;
+  }
+  (void)E;
+  for (int a = 0; a < 3; ++a) {
+    const int rc = io_full(rd, fd, h + a * T, bytes, foff + a * stride, msg);
+    if (rc != RATEL_OK) return rc;
+  }
+  return RATEL_OK;
+}
+
 #define SK(call)                                                                                         \
   do {                                                                                                   \
     cudaError_t e_ = (call);                                                                             \
@@ -777,8 +796,8 @@ int ssd_run_job_cpu(SsdEngine& E, Block& B, std::string& msg) {
       const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
       disk_acquire(E);
       const double t0 = now_s();
-      for (int a = 0; a < 3; ++a) {
-        const int rc = io_full(true, f.fd, h + a * T, bytes, f.off + a * f.stride + off * 4, msg);
+      {
+        const int rc = io_tile(E, E.rd_ring, true, f.fd, h, T, bytes, f.off + off * 4, f.stride, msg);
         if (rc != RATEL_OK) {
           disk_release(E, false);
           return rc;
@@ -859,8 +878,8 @@ int ssd_run_job(SsdEngine& E, const SsdJob& job, std::string& msg) {
       const uint64_t bytes = (len * 4 + kSsdAlign - 1) / kSsdAlign * kSsdAlign;
       disk_acquire(E);
       const double t0 = now_s();
-      for (int a = 0; a < 3; ++a) {
-        const int rc = io_full(true, f.fd, h + a * T, bytes, f.off + a * f.stride + off * 4, msg);
+      {
+        const int rc = io_tile(E, E.rd_ring, true, f.fd, h, T, bytes, f.off + off * 4, f.stride, msg);
         if (rc != RATEL_OK) {
           disk_release(E, false);
           return rc;
@@ -999,8 +1018,8 @@ void ssd_writer_main(SsdEngine* E) {
       }
       const float* h = E->h_ring + 3ull * t.slot * T;
       const double t0 = now_s();
-      for (int a = 0; a < 3 && rc == RATEL_OK; ++a)
-        rc = io_full(false, t.fd, const_cast<float*>(h + a * T), t.bytes, t.foff + a * t.stride, m);
+      if (rc == RATEL_OK)
+        rc = io_tile(*E, E->wr_ring, false, t.fd, const_cast<float*>(h), T, t.bytes, t.foff, t.stride, m);
       E->write_s += now_s() - t0;
       E->write_bytes += 3 * t.bytes;
       if (ssd_simplex()) disk_release(*E, false);
@@ -1018,6 +1037,14 @@ void ssd_writer_main(SsdEngine* E) {
 int ssd_create() {
   SsdEngine* E = new SsdEngine();
   G.ssd = E;  // destroy_all() tears down whatever was created
+  if (G.cfg.ssd_io == RATEL_SSD_IO_URING) {
+    for (IoRing* r : {&E->rd_ring, &E->wr_ring}) {
+      const int e = r->open_ring(32);
+      if (e != 0)
+        return set_error(RATEL_EIO, "ratel_register_block: cfg.ssd_io = RATEL_SSD_IO_URING but io_uring_setup "
+                                    "failed: %s", strerror(-e));
+    }
+  }
   const size_t n = static_cast<size_t>(G.cfg.pipeline_depth) * 3 * G.cfg.tile_elems;
   CK(cudaHostAlloc(&E->h_ring, n * sizeof(float), cudaHostAllocDefault));
   CK(cudaMalloc(&E->d_ring, n * sizeof(float)));
@@ -1228,6 +1255,7 @@ int validate_config(const ratel_config& c) {
     return set_error(RATEL_EINVAL, "cfg.k1_kernel");
   if (c.ssd_schedule != RATEL_SSD_DUPLEX && c.ssd_schedule != RATEL_SSD_SIMPLEX)
     return set_error(RATEL_EINVAL, "cfg.ssd_schedule");
+  if (c.ssd_io != RATEL_SSD_IO_PREAD && c.ssd_io != RATEL_SSD_IO_URING) return set_error(RATEL_EINVAL, "cfg.ssd_io");
   return RATEL_OK;
 }
 
@@ -1385,6 +1413,7 @@ void ratel_default_config(ratel_config* cfg) {
   cfg->cta_tiles = 0;
   cfg->k1_kernel = RATEL_UPDATE_TMA;
   cfg->ssd_schedule = RATEL_SSD_DUPLEX;
+  cfg->ssd_io = RATEL_SSD_IO_PREAD;
 }
 
 uint64_t ratel_padded_numel(uint64_t numel, int world_size) {

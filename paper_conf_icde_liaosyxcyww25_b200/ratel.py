@@ -43,6 +43,8 @@ RATEL_UPDATE_LDG = 1
 RATEL_UPDATE_LDG_LITE = 2
 RATEL_SSD_DUPLEX = 0
 RATEL_SSD_SIMPLEX = 1
+RATEL_SSD_IO_PREAD = 0
+RATEL_SSD_IO_URING = 1
 RATEL_MAX_BLOCKS = 4096
 RATEL_MAX_RANGES_PER_BLOCK = 32
 
@@ -72,6 +74,7 @@ class ratel_config(ctypes.Structure):
         ("cta_tiles", ctypes.c_int),
         ("k1_kernel", ctypes.c_int),
         ("ssd_schedule", ctypes.c_int),
+        ("ssd_io", ctypes.c_int),
     ]
 
 

@@ -117,9 +117,10 @@ def test_generator_keys_match_synth():
 
 
 def test_struct_layouts_match_header():
-    # ratel_config: int, double, int, int, uint64, int x 7 -> 64 bytes
-    assert ctypes.sizeof(R.ratel_config) == 64
+    # ratel_config: int, double, int, int, uint64, int x 9 -> 68 bytes, padded to 72 (double alignment)
+    assert ctypes.sizeof(R.ratel_config) == 72
     assert R.ratel_config.k1_kernel.offset == 56
+    assert R.ratel_config.ssd_schedule.offset == 60 and R.ratel_config.ssd_io.offset == 64
     assert R.ratel_config.update_streams.offset == 48
     assert R.ratel_config.tile_elems.offset == 24
     # ratel_range: 2 ptrs, int, 3 ptrs, uint64, int -> 64 bytes
@@ -134,3 +135,28 @@ def test_ssd_range_bytes():
         want = 3 * ((4 * (e - b) + 4095) // 4096 * 4096)
         assert R.ratel_ssd_range_bytes(n, world, rank) == want
     assert R.ratel_ssd_range_bytes(10, 0, 0) == 0
+
+
+def test_struct_layouts_match_the_c_compiler(tmp_path):
+    """ratel.py's ctypes structs against what a C compiler makes of
+    include/ratel.h (sizeof / offsetof of every field)."""
+    import subprocess
+    fields = {"ratel_config": [f[0] for f in R.ratel_config._fields_],
+              "ratel_range": [f[0] for f in R.ratel_range._fields_]}
+    src = ["#include <stdio.h>", "#include <stddef.h>", '#include "ratel.h"', "int main(void) {"]
+    for st, fs in fields.items():
+        src.append(f'  printf("{st} size %zu\\n", sizeof({st}));')
+        for f in fs:
+            src.append(f'  printf("{st} {f} %zu\\n", offsetof({st}, {f}));')
+    src += ["  return 0;", "}"]
+    c = tmp_path / "layout.c"
+    c.write_text("\n".join(src))
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-I", os.path.join(ROOT, "include"), "-o", str(exe), str(c)])
+    out = subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split("\n")
+    got = {tuple(line.split()[:2]): int(line.split()[2]) for line in out if line.strip()}
+    for st, fs in fields.items():
+        cls = getattr(R, st)
+        assert got[(st, "size")] == ctypes.sizeof(cls), st
+        for f in fs:
+            assert got[(st, f)] == getattr(cls, f).offset, (st, f)

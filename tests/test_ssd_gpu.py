@@ -210,3 +210,23 @@ def test_ssd_simplex_schedule_bitwise(cuda_dev, tmp_path, cpu):
     assert_bitwise(snapshot(ssd), snapshot(ref))
     for b in ssd:
         b.close()
+
+
+@pytest.mark.parametrize("cpu,schedule", [(False, 0), (True, 0), (False, 1)])
+def test_ssd_io_uring_bitwise(cuda_dev, tmp_path, cpu, schedule):
+    """cfg.ssd_io = RATEL_SSD_IO_URING (each I/O thread keeps up to 32 requests
+    of <= 4 MiB in flight through its own io_uring) moves the same bytes as
+    pread/pwrite: bitwise the device / HOST_COMPUTE result, with clipping, the
+    simplex schedule and one state file for all blocks."""
+    base, ssd = 0, []
+    for i, n in enumerate(SIZES):
+        b = SsdBlock(i, [n], cuda_dev, tmp_path / "states.bin", base=base, cpu=cpu)
+        base = b.file_bytes
+        ssd.append(b)
+    run(ssd, 3, max_norm=1e-3, tile_elems=TILE, pipeline_depth=3, ssd_io=R.RATEL_SSD_IO_URING,
+        ssd_schedule=schedule, host_threads=4)
+    ref = [GpuBlock(i, [n], cuda_dev, host_compute=cpu) for i, n in enumerate(SIZES)]
+    run(ref, 3, max_norm=1e-3, host_threads=4)
+    assert_bitwise(snapshot(ssd), snapshot(ref))
+    for b in ssd:
+        b.close()

@@ -106,6 +106,9 @@ def main():
     ap.add_argument("--schedules", default="duplex,simplex",
                     help="cfg.ssd_schedule: duplex (reader and writer free) and/or simplex (the paper's Fig. 3b "
                          "order: one transfer at a time, write-back of tile k after the read of tile k+1)")
+    ap.add_argument("--io", default="pread",
+                    help="cfg.ssd_io: pread (one blocking request at a time) and/or uring (io_uring, up to 32 "
+                         "requests of 4 MiB in flight per I/O thread)")
     args = ap.parse_args()
 
     import torch
@@ -117,12 +120,13 @@ def main():
     dev = torch.device("cuda:0")
     sizes = model_blocks(args.shape)[:args.blocks]
     path = os.path.join(args.dir, "ratel_ssd_states.bin")
-    runs = [(d, h, sc) for h in args.handlers.split(",") for d in (int(x) for x in args.depths.split(","))
-            for sc in args.schedules.split(",")]
-    for depth, handler, sched in runs:
+    runs = [(d, h, sc, io) for h in args.handlers.split(",") for d in (int(x) for x in args.depths.split(","))
+            for sc in args.schedules.split(",") for io in args.io.split(",")]
+    for depth, handler, sched, io in runs:
         cfg = R.ratel_default_config()
         cfg.pipeline_depth = depth
         cfg.ssd_schedule = {"duplex": R.RATEL_SSD_DUPLEX, "simplex": R.RATEL_SSD_SIMPLEX}[sched]
+        cfg.ssd_io = {"pread": R.RATEL_SSD_IO_PREAD, "uring": R.RATEL_SSD_IO_URING}[io]
         if args.tile_elems:
             cfg.tile_elems = args.tile_elems
         R.ratel_init(0, 0, 1, None, cfg)
@@ -181,7 +185,7 @@ def main():
             gbs = 24.0 * P / dt / 1e9
             print(json.dumps({
                 "residency": "ssd" if handler == "gpu" else "ssd_host_compute", "shape": args.shape, "blocks": len(sizes), "params": P,
-                "pipeline_depth": depth, "schedule": sched, "tile_elems": int(cfg.tile_elems), "steps": args.steps,
+                "pipeline_depth": depth, "schedule": sched, "io": io, "tile_elems": int(cfg.tile_elems), "steps": args.steps,
                 "warmup": args.warmup, "ms_per_step": dt * 1e3, "params_per_s": P / dt,
                 "ssd_gbs_24B_per_param": gbs, "roofline_gbs": probe.get("roofline_gbs"),
                 "frac": gbs / probe["roofline_gbs"] if probe.get("roofline_gbs") else None,
