@@ -103,7 +103,7 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory, data_parallel="fus
                                     for r in ranges])
                 if t == 0 and data_parallel == "fused":   # this rank's view of the peer's G16
                     dist.barrier()
-                    q = 1 - rank
+                    q = (rank + 1) % world
                     peer_view = []
                     for r in ranges:
                         ptr = r.peer_g16[q]
@@ -170,15 +170,16 @@ def _diagnose(init, res, world, k, got):
     return out
 
 
-@pytest.mark.parametrize("peer_memory,data_parallel", [("ipc", "fused"), ("symm", "fused"), ("symm", "reduced")])
-def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_parallel):
+@pytest.mark.parametrize("peer_memory,data_parallel,world", [("ipc", "fused", 2), ("symm", "fused", 2),
+                                                             ("symm", "reduced", 2), ("ipc", "fused", 4)])
+def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_parallel, world):
     """peer_memory="symm" (torch symmetric memory) needs a GPU per rank; on a
     one-GPU box only the CUDA-IPC mapping runs.  data_parallel="reduced": both
     ranks see the same micro-batch (identical gradients, R11), the library only
     all-gathers P16 over NCCL -- the mean of identical gradients is the same
     step, so the same oracle check applies."""
     n = torch.cuda.device_count()
-    world, shared = (2, n < 2)
+    shared = n < world
     if shared and peer_memory == "symm" and data_parallel == "fused":
         pytest.skip("torch symmetric memory refuses ranks that share a GPU")
     ctx = torch.multiprocessing.get_context("spawn")
@@ -202,12 +203,14 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_par
     assert all(p.exitcode == 0 for p in procs), [p.exitcode for p in procs]
     init = res[0][0]
     # the hand-off order (each hand-off is a barrier on the library's communicator) is the same on both ranks
-    assert [h[0] for h in res[0][5]] == [h[0] for h in res[1][5]], (res[0][5], res[1][5])
+    for q in range(1, world):
+        assert [h[0] for h in res[0][5]] == [h[0] for h in res[q][5]], (res[0][5], res[q][5])
     for q in range(world if data_parallel == "fused" else 0):   # the mapping of the peer's G16
         for k in range(len(init)):
-            assert np.array_equal(res[q][4][k], res[1 - q][1][0][k]), ("peer view", q, k)
+            assert np.array_equal(res[q][4][k], res[(q + 1) % world][1][0][k]), ("peer view", q, k)
     for k in range(len(init)):
-        assert np.array_equal(res[1][0][k], init[k])          # same model on both ranks
+        for q in range(1, world):
+            assert np.array_equal(res[q][0][k], init[k])      # the same model on every rank
     wd = [1, 0] * NB                                           # weights decay, biases / LN do not
     refs = [oracle.Range.fresh(a.astype(np.float32), wd[k]) for k, a in enumerate(init)]
     for t in range(STEPS):
@@ -222,6 +225,7 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_par
             check_range(got, ref, own_rne=oracle.bf16_rne, what=f"api dp range {k}")
         except AssertionError as e:
             raise AssertionError(f"{e}; closest hypothesis: {_diagnose(init, res, world, k, got)}") from None
-        assert np.array_equal(res[1][2][k]["p16"], res[0][2][k]["p16"])
+        for q in range(1, world):
+            assert np.array_equal(res[q][2][k]["p16"], res[0][2][k]["p16"])
         for q in range(world):                                 # resume: P16 rebuilt from the masters
             assert np.array_equal(res[q][3][k], oracle.bf16_rne(got["p32"])), (k, q)

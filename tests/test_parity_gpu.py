@@ -506,6 +506,10 @@ def test_range_beyond_2pow32_elements_sampled_vs_oracle(cuda_dev):
                    p16=torch_to_u16(p[ii]))
         check_range(got, ref, own_rne=oracle.bf16_rne, what="2^32+ range")
         assert np.array_equal(got["p16"], oracle.bf16_rne(got["p32"]))
+        # the P16 refresh (64-bit grid-stride indexing) over the same 2^32+ range
+        p.fill_(2.0)
+        R.ratel_refresh_params(0, None)
+        assert np.array_equal(torch_to_u16(p[ii]), got["p16"])
     del th, m, v, p, g
     torch.cuda.empty_cache()
 
