@@ -70,7 +70,7 @@
 extern "C" {
 #endif
 
-#define RATEL_ABI_VERSION 1
+#define RATEL_ABI_VERSION 2   /* 2: ratel_config gained ssd_schedule and ssd_io (72 bytes) */
 #define RATEL_MAX_BLOCKS 4096          /* block ids are 0 .. RATEL_MAX_BLOCKS-1 */
 #define RATEL_MAX_RANGES_PER_BLOCK 32
 
