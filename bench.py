@@ -19,8 +19,16 @@ Printed: ONE JSON line on rank 0.
              states: 24 B/param over the host link vs this run's duplex
              probe; HOST_COMPUTE: 32 B/param of host DRAM vs this run's
              host_stream probe -- K1's numbers then under roofline.k1)
-  cpu_baseline  the CPU oracle on a bounded sample, on this host's cores
-`--impl reference` times the oracle as the reference arm.
+  cpu_baseline  the CPU oracle on a whole 13B block per pass, on this host's cores
+  overlap    (N=1) device-resident C2 sweep, 1K-64K tokens: AGO vs deferred vs
+             backward alone, 3 bracketed repetitions, NVML energy
+  overlap_host / overlap_hostcompute  (N=1) pinned-host states of 16 x 13B
+             blocks, per-tensor hand-off, 32K-192K tokens, 3 bracketed reps
+  multi_gpu  (N>1) NCCL all-gather busbw at the C3 / workload slices, the 8-byte
+             allreduce latency, all-rank host-link probe, all-rank P16 equality,
+             NCCL init log summary; roofline.nvlink and roofline.step_bounds_ms
+`--impl reference` times the oracle as the reference arm.  `--gpus N` outside
+torchrun re-launches this script under torch.distributed.run (N ranks).
 """
 from __future__ import annotations
 
