@@ -1116,6 +1116,15 @@ def run_e2e(args, R, torch, dev, dev_index, rank, world):
 
 
 # ------------------------------------------------------------------- main
+def token_list(x: str):
+    """--overlap-sweep / --overlap-host-sweep: comma-separated token counts;
+    '', '0' or 'none' disables the probe."""
+    x = x.strip().strip("'\"")
+    if x.lower() in ("", "0", "none"):
+        return []
+    return [int(v) for v in x.split(",") if v]
+
+
 def free_port() -> int:
     import socket
     with socket.socket() as so:
@@ -1270,13 +1279,13 @@ def main():
     ap.add_argument("--share-gpu", action="store_true",
                     help="test mode: every rank on cuda:0 with real NCCL (each rank its own NCCL host id, "
                          "loopback sockets); numbers are plumbing, not a scaling result")
-    ap.add_argument("--overlap-sweep", type=lambda x: [int(v) for v in x.split(",") if v], default=[1024, 2048, 8192, 32768, 65536],
+    ap.add_argument("--overlap-sweep", type=token_list, default=[1024, 2048, 8192, 32768, 65536],
                     help="device-resident AGO vs deferred overlap sweep: tokens per step, comma-separated "
-                         "('' disables)")
+                         "(0 disables)")
     ap.add_argument("--overlap-reps", type=int, default=3, help="alternating repetitions per overlap point")
-    ap.add_argument("--overlap-host-sweep", type=lambda x: [int(v) for v in x.split(",") if v],
+    ap.add_argument("--overlap-host-sweep", type=token_list,
                     default=[32768, 65536, 98304, 131072, 196608],
-                    help="pinned-host per-tensor AGO overlap probe: tokens per step, comma-separated ('' disables)")
+                    help="pinned-host per-tensor AGO overlap probe: tokens per step, comma-separated (0 disables)")
     ap.add_argument("--overlap-host-blocks", type=int, default=16,
                     help="13B-shape blocks of pinned-host states in the host overlap probe (16 = 5.0B params, 60 GB)")
     ap.add_argument("--arm", default="before", choices=["before", "after"],

@@ -7,7 +7,7 @@ set -u
 mkdir -p gpurun_out
 out=gpurun_out/configs.jsonl
 : > $out
-common="--no-e2e --no-cpu-baseline --overlap-tokens 0 --overlap-host-tokens 0"
+common="--no-e2e --no-cpu-baseline --overlap-sweep 0 --overlap-host-sweep 0"
 run() { timeout 900 python bench.py "$@" $common 2> gpurun_out/configs_err.log | tail -n 1 >> $out; }
 run --shape 30B --blocks 12 --clip 1.0 --steps 20 --warmup 3
 run --shape 70B --residency host --blocks 3 --steps 3 --warmup 3

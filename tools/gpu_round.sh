@@ -12,10 +12,10 @@ timeout 900  python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/
 # launch list of the bench command (cold-cache, serialised: compare shares)
 timeout 900  ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none \
              --csv --log-file gpurun_out/launches.csv \
-             python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu-baseline --overlap-tokens 0 --overlap-host-tokens 0 > gpurun_out/ncu_launch.log 2>&1
+             python bench.py --steps 2 --warmup 1 --no-e2e --no-cpu-baseline --overlap-sweep 0 --overlap-host-sweep 0 > gpurun_out/ncu_launch.log 2>&1
 # one full capture of K1 on a 13B block
 timeout 900  ncu --set full --clock-control none --import-source on -k regex:adam_update -s 4 -c 1 -o gpurun_out/k1_full \
-             python bench.py --blocks 4 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --overlap-tokens 0 --overlap-host-tokens 0 > gpurun_out/ncu_full.log 2>&1
+             python bench.py --blocks 4 --steps 1 --warmup 1 --no-e2e --no-cpu-baseline --overlap-sweep 0 --overlap-host-sweep 0 > gpurun_out/ncu_full.log 2>&1
 for tool in memcheck racecheck synccheck initcheck; do
   timeout 900 compute-sanitizer --tool $tool --kernel-name kns=ratel --print-limit 10 python tools/sanitize_run.py \
               > gpurun_out/sanitizer_$tool.log 2>&1

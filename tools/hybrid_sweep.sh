@@ -5,5 +5,5 @@
 mkdir -p gpurun_out; : > gpurun_out/hybrid.jsonl
 for f in ${FRACS:-0 0.2 0.3 0.4 0.5 0.6 1}; do
   timeout 600 python bench.py --shape 13B --residency hybrid --hybrid-gpu-frac $f --blocks 8 --steps 3 --warmup 3 \
-      --no-e2e --no-cpu-baseline --overlap-tokens 0 --overlap-host-tokens 0 2>>gpurun_out/hybrid.err | tail -n 1 >> gpurun_out/hybrid.jsonl
+      --no-e2e --no-cpu-baseline --overlap-sweep 0 --overlap-host-sweep 0 2>>gpurun_out/hybrid.err | tail -n 1 >> gpurun_out/hybrid.jsonl
 done

@@ -10,8 +10,8 @@ ROUNDS=${ROUNDS:-3}
 for r in $(seq 1 "$ROUNDS"); do
   for v in approx ieee; do
     if [ "$v" = ieee ]; then export RATEL_LIB=build/variants/libratel_ieee.so; else unset RATEL_LIB; fi
-    line=$(python bench.py --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --overlap-sweep '' \
-           --overlap-host-sweep '' 2>/dev/null | grep '^{')
+    line=$(python bench.py --steps 20 --warmup 5 --no-e2e --no-cpu-baseline --overlap-sweep 0 \
+           --overlap-host-sweep 0 2>/dev/null | grep '^{')
     python - "$v" "$r" "$line" >> "$OUT" <<'PY'
 import json, sys
 v, r, line = sys.argv[1], int(sys.argv[2]), json.loads(sys.argv[3])
