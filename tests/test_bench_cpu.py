@@ -136,3 +136,38 @@ def test_nccl_log_summary(tmp_path, monkeypatch):
     out = bench.nccl_init_summary()
     assert out["log"] == str(log) and len(out["lines"]) == 3
     assert any("via P2P" in line for line in out["lines"]) and any("NVLS" in line for line in out["lines"])
+
+
+def test_bench_host_helpers(monkeypatch, tmp_path):
+    """Host-side helpers added for N > 1 and the reference arm: the sweep
+    parser, the WORLD_SIZE / --gpus reconciliation, the NCCL log routing and
+    the CPU facts reported with the oracle."""
+    import argparse
+    sys.path.insert(0, ROOT)
+    import bench
+    assert bench.token_list("0") == [] and bench.token_list("") == [] and bench.token_list("none") == []
+    assert bench.token_list("1024,2048") == [1024, 2048]
+    monkeypatch.setenv("WORLD_SIZE", "4")
+    assert bench.relaunch_or_world(argparse.Namespace(gpus=None)) == 4
+    assert bench.relaunch_or_world(argparse.Namespace(gpus=4)) == 4
+    try:
+        bench.relaunch_or_world(argparse.Namespace(gpus=2))
+        raise AssertionError("a --gpus / WORLD_SIZE mismatch must exit")
+    except SystemExit as e:
+        assert e.code == 2
+    monkeypatch.delenv("WORLD_SIZE")
+    assert bench.relaunch_or_world(argparse.Namespace(gpus=None)) == 1
+    assert bench.relaunch_or_world(argparse.Namespace(gpus=1)) == 1
+    monkeypatch.delenv("NCCL_DEBUG_FILE", raising=False)
+    monkeypatch.delenv("NCCL_DEBUG", raising=False)
+    monkeypatch.setattr(bench, "NCCL_LOG_DIR", str(tmp_path / "logs"))
+    bench.nccl_log_env()
+    assert os.environ["NCCL_DEBUG"] == "INFO" and "%p" in os.environ["NCCL_DEBUG_FILE"]
+    assert os.path.isdir(tmp_path / "logs")
+    facts = bench.cpu_facts()
+    assert {"cpu_model", "sockets", "numa_nodes", "nproc"} <= set(facts) and facts["nproc"] >= 1
+    monkeypatch.setenv("NCCL_HOSTID", "x")
+    for k in ("NCCL_SOCKET_IFNAME", "NCCL_IB_DISABLE", "NCCL_DEBUG_SUBSYS"):
+        monkeypatch.delenv(k, raising=False)          # restored after the test
+    bench.share_gpu_nccl_env(3)
+    assert os.environ["NCCL_HOSTID"] == "ratel-bench-rank3"
