@@ -145,6 +145,8 @@ def test_bench_host_helpers(monkeypatch, tmp_path):
     import argparse
     sys.path.insert(0, ROOT)
     import bench
+    for k in ("NCCL_SOCKET_IFNAME", "NCCL_IB_DISABLE", "NCCL_DEBUG_SUBSYS", "NCCL_DEBUG", "NCCL_DEBUG_FILE"):
+        monkeypatch.delenv(k, raising=False)          # whatever the helpers set is undone after the test
     assert bench.token_list("0") == [] and bench.token_list("") == [] and bench.token_list("none") == []
     assert bench.token_list("1024,2048") == [1024, 2048]
     monkeypatch.setenv("WORLD_SIZE", "4")
@@ -158,8 +160,6 @@ def test_bench_host_helpers(monkeypatch, tmp_path):
     monkeypatch.delenv("WORLD_SIZE")
     assert bench.relaunch_or_world(argparse.Namespace(gpus=None)) == 1
     assert bench.relaunch_or_world(argparse.Namespace(gpus=1)) == 1
-    monkeypatch.delenv("NCCL_DEBUG_FILE", raising=False)
-    monkeypatch.delenv("NCCL_DEBUG", raising=False)
     monkeypatch.setattr(bench, "NCCL_LOG_DIR", str(tmp_path / "logs"))
     bench.nccl_log_env()
     assert os.environ["NCCL_DEBUG"] == "INFO" and "%p" in os.environ["NCCL_DEBUG_FILE"]
@@ -167,7 +167,5 @@ def test_bench_host_helpers(monkeypatch, tmp_path):
     facts = bench.cpu_facts()
     assert {"cpu_model", "sockets", "numa_nodes", "nproc"} <= set(facts) and facts["nproc"] >= 1
     monkeypatch.setenv("NCCL_HOSTID", "x")
-    for k in ("NCCL_SOCKET_IFNAME", "NCCL_IB_DISABLE", "NCCL_DEBUG_SUBSYS"):
-        monkeypatch.delenv(k, raising=False)          # restored after the test
     bench.share_gpu_nccl_env(3)
     assert os.environ["NCCL_HOSTID"] == "ratel-bench-rank3"
