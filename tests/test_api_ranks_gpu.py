@@ -57,7 +57,7 @@ def _flat_ranges(model):
     return out
 
 
-def _rank_main(rank, world, shared, port, res_q, peer_memory, data_parallel="fused"):
+def _rank_main(rank, world, shared, port, res_q, peer_memory, data_parallel="fused", residency="device"):
     if shared:
         os.environ["NCCL_HOSTID"] = f"ratel-api-rank{rank}"
         os.environ["NCCL_SOCKET_IFNAME"] = "lo"
@@ -91,7 +91,7 @@ def _rank_main(rank, world, shared, port, res_q, peer_memory, data_parallel="fus
             opt = Ratel_Optimizer([list(b.parameters()) for b in model], lr=HPK["lr"],
                                   betas=(HPK["beta1"], HPK["beta2"]), eps=HPK["eps"],
                                   weight_decay=HPK["weight_decay"], data_parallel=data_parallel,
-                                  peer_memory=peer_memory)
+                                  peer_memory=peer_memory, residency=residency)
             Ratel_hook(opt)
             ranges = [r for rs in opt.blocks for r in rs]
             local_grads = []
@@ -170,9 +170,10 @@ def _diagnose(init, res, world, k, got):
     return out
 
 
-@pytest.mark.parametrize("peer_memory,data_parallel,world", [("ipc", "fused", 2), ("symm", "fused", 2),
-                                                             ("symm", "reduced", 2), ("ipc", "fused", 4)])
-def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_parallel, world):
+@pytest.mark.parametrize("peer_memory,data_parallel,world,residency", [
+    ("ipc", "fused", 2, "device"), ("symm", "fused", 2, "device"), ("symm", "reduced", 2, "device"),
+    ("ipc", "fused", 4, "device"), ("ipc", "fused", 2, "host")])
+def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_parallel, world, residency):
     """peer_memory="symm" (torch symmetric memory) needs a GPU per rank; on a
     one-GPU box only the CUDA-IPC mapping runs.  data_parallel="reduced": both
     ranks see the same micro-batch (identical gradients, R11), the library only
@@ -185,7 +186,8 @@ def test_paper_api_data_parallel_fused_vs_oracle(cuda_dev, peer_memory, data_par
     ctx = torch.multiprocessing.get_context("spawn")
     res_q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, res_q, peer_memory, data_parallel))
+    procs = [ctx.Process(target=_rank_main, args=(r, world, shared, port, res_q, peer_memory, data_parallel,
+                                                              residency))
              for r in range(world)]
     for p in procs:
         p.start()
